@@ -1,0 +1,333 @@
+#!/usr/bin/env python3
+"""bench.py -- headline benchmark of the sdag hot path on B200.
+
+Workload (BASELINE.json configs[1]): 25-point radius-4 FP64 Laplacian,
+512^3 grid per GPU, one sweep per step.  At N GPUs the grid is weak-scaled
+as z-slabs (512N x 512 x 512) with a per-step NCCL halo exchange (a7).
+A step = parse/plan done once up front (a1-a3, host), then one sweep
+(a4-a5) [+ exchange (a7) for N>1] over the resident input.
+
+Prints ONE JSON line (rank 0).  --impl reference times the CPU oracle (the
+reference arm of this tier) on the same metric/config.  --config selects
+another BASELINE stencil for reporting (not the headline line).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "FP64 GFLOP/s and HBM GB/s per stencil, % of roofline, at 1/2/4/8 B200"
+
+CONFIGS = {
+    # name: (spec, dims per GPU, BASELINE config string, flops/pt)
+    "lap25": ("lap25", (512, 512, 512), "3D 4th-order 25-point Laplacian (order 4), 512^3 FP64, single GPU"),
+    "jacobi7": ("jacobi7", (64, 64, 64), "3D 7-point Jacobi (order 1), 64^3 FP64 grid, single sweep, 1 input/1 output"),
+    "hypterm": ("hypterm", (320, 320, 320), "ExpCNS hypterm-style DAG (order 4, ~8 inputs, multiple outputs), 320^3 FP64"),
+    "rhs4center": ("rhs4center", (320, 320, 320),
+                   "SW4 rhs4th3fort-style elastic-wave stencil (order 2, multi-statement, ~300 FLOP/pt), 320^3 FP64"),
+    "smooth27": ("smooth27", (1024, 1024, 1024),
+                 "iterated 27-point order-2 stencil, 1024^3 FP64 weak-scaled as z-slabs with halo exchange"),
+}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d.get("hbm_gbs", 6650.0), "measured"
+    return 6650.0, "fallback"
+
+
+def load_traffic(variant):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        d = json.load(f)
+    return d.get(variant)
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+
+    def __init__(self, index):
+        self.index = index
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            p = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                  "-lms", "100"], stdout=subprocess.PIPE, text=True)
+        except Exception:
+            return
+        while not self._stop.is_set():
+            line = p.stdout.readline()
+            if not line:
+                break
+            self.samples.append([x.strip() for x in line.split(",")])
+        p.terminate()
+        try:
+            p.wait(timeout=2)
+        except Exception:
+            p.kill()
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        time.sleep(0.3)
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=3)
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for s in self.samples:
+            for n, v in zip(names, s[3:7]):
+                if v.strip().lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.samples)}
+
+
+def cpu_baseline_lap25(A, c, seconds=10.0):
+    """Time the oracle (as it stands) on a bounded z-slab sample of the same input."""
+    import oracle
+    cores = len(os.sched_getaffinity(0))
+    nz, ny, nx = A.shape
+    planes = 32
+    out = np.zeros_like(A)
+    oracle.lap25(A, c, out=out, krange=(4, 4 + 2))  # warm (build + page-in)
+    reps, t0 = 0, time.perf_counter()
+    k0 = 4
+    while True:
+        oracle.lap25(A, c, out=out, krange=(k0, k0 + planes))
+        reps += 1
+        k0 = 4 + (k0 + planes - 4) % (nz - 8 - planes)
+        if time.perf_counter() - t0 >= seconds:
+            break
+    dt = time.perf_counter() - t0
+    pts = reps * planes * (ny - 8) * (nx - 8)
+    return {"value": pts * 29 / dt / 1e9, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
+            "sample": f"{reps} x {planes}-plane z-slabs of the 512^3 input ({pts} interior points), "
+                      f"{dt:.1f} s, OpenMP over k"}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle on the host cores, same metric/config."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import synth
+    dims = CONFIGS["lap25"][1]
+    ins, sc = synth.lap25_inputs(dims)
+    A = ins["A"]
+    c = [sc[k] for k in ("c0", "c1", "c2", "c3", "c4")]
+    import oracle
+    cores = len(os.sched_getaffinity(0))
+    out = np.zeros_like(A)
+    planes = 16
+    nz, ny, nx = dims
+    oracle.lap25(A, c, out=out, krange=(4, 6))
+    for _ in range(args.warmup):
+        oracle.lap25(A, c, out=out, krange=(4, 4 + planes))
+    t0 = time.perf_counter()
+    for s in range(args.steps):
+        k0 = 4 + (s * planes) % (nz - 8 - planes)
+        oracle.lap25(A, c, out=out, krange=(k0, k0 + planes))
+    dt = time.perf_counter() - t0
+    pts = args.steps * planes * (ny - 8) * (nx - 8)
+    val = pts * 29 / dt / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "GFLOP/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": CONFIGS["lap25"][2], "stencil": "lap25", "grid": list(dims),
+                       "step": f"oracle sweep of a {planes}-plane z-slab sample (bounded CPU time)"},
+            "cpu_baseline": {"value": val, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
+                             "sample": f"{args.steps} steps x {planes} planes x {ny - 8}x{nx - 8} interior points"},
+            "e2e": {"value": val, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="sdag", choices=["sdag", "reference"])
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--variant", default=None)
+    ap.add_argument("--tune", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(3, args.warmup)
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import paper_conf_ipps_rawatvsrps19_b200 as sdag
+    import synth
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as tdist
+        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dist = tdist
+    name = "lap25"
+    spec = sdag.spec_text(name)
+    ldims = CONFIGS[name][1]
+    gdims = (ldims[0] * world, ldims[1], ldims[2])
+    ins, sc = synth.lap25_inputs(ldims, cfg="cfg2") if world == 1 else (None, dict(synth.LAP25_COEFS))
+    c = [sc[k] for k in ("c0", "c1", "c2", "c3", "c4")]
+    stream = torch.cuda.current_stream()
+
+    if world == 1:
+        plan = sdag.Plan(spec, ldims, tune=args.tune, variant=args.variant)
+        A = ins["A"]
+        dA = torch.from_numpy(A).cuda()
+        dB = torch.zeros(ldims, dtype=torch.float64, device="cuda")
+        arrays = [dB, dA]
+        info = plan.info
+        pts_rank = info["points"]
+
+        def step():
+            plan.apply(arrays, scalars=c, stream=stream)
+    else:
+        uid = [sdag.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        comm = sdag.nccl_comm_create(uid[0], world, rank, local)
+        dd = sdag.Dist(spec, gdims, rank, world, comm=comm, tune=args.tune, variant=args.variant)
+        (nza, ny, nx), g0 = dd.layout()
+        part = sdag.slab_partition(gdims[0], 4, world, rank)
+        # this rank's slab of the global synthetic input, regenerated from the counter-based generator
+        full = synth.uniform((nza, ny, nx), -1.0, 1.0, "cfg2-slab", rank)
+        dA = torch.from_numpy(full).cuda()
+        dB = torch.zeros((nza, ny, nx), dtype=torch.float64, device="cuda")
+        arrays = [dB, dA]
+        plan = dd.plan
+        info = plan.info
+        pts_rank = (part["k_hi"] - part["k_lo"]) * (ny - 8) * (nx - 8)
+        comm_stream = torch.cuda.Stream()
+
+        def step():
+            dd.apply(arrays, scalars=c, stream=stream, comm_stream=comm_stream)
+
+    flops_pt = info["flops_per_point"]
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    l0 = sdag.launch_count()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with Clocks(local) as clk:
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(args.steps):
+            step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+    launches = sdag.launch_count() - l0
+    ms = e0.elapsed_time(e1)
+    ms_t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    pts_t = torch.tensor([float(pts_rank)], dtype=torch.float64, device="cuda")
+    if dist:
+        dist.barrier()
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(pts_t, op=dist.ReduceOp.SUM)
+    ms_max = float(ms_t.item())
+    total_pts = float(pts_t.item())
+    gflops = total_pts * flops_pt * args.steps / (ms_max * 1e-3) / 1e9
+
+    # dominant kernel: the sweep.  N=1: the step is exactly one launch.  N>1: time the
+    # local sweep kernel alone (same stream, same launch configuration).
+    kms = ms / max(1, launches) if world == 1 else None
+    if world > 1:
+        ka, kb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        lp = dd.plan
+        ka.record(stream)
+        for _ in range(args.steps):
+            lp.apply(arrays, scalars=c, stream=stream)
+        kb.record(stream)
+        torch.cuda.synchronize()
+        kms = ka.elapsed_time(kb) / args.steps
+    peak, peak_src = load_peaks()
+    bytes_launch = info["bytes_per_point"] * info["points"]
+    achieved = bytes_launch / (kms * 1e-3) / 1e9
+    traffic = load_traffic(info["variant"])
+
+    e2e = None
+    if not args.no_e2e and world == 1:
+        hA = torch.from_numpy(A).pin_memory().numpy()
+        hB = torch.zeros(ldims, dtype=torch.float64).pin_memory().numpy()
+        ee = []
+        plan.apply_host([hB, hA], scalars=c, stream=stream)  # warm workspace
+        up = down = 0
+        for _ in range(max(3, min(args.steps, 5))):
+            t0 = time.perf_counter()
+            up, down = plan.apply_host([hB, hA], scalars=c, stream=stream)
+            ee.append(time.perf_counter() - t0)
+        t_e2e = statistics.median(ee)
+        e2e = {"value": info["points"] * flops_pt / t_e2e / 1e9, "unit": "GFLOP/s", "h2d_bytes_per_step": up,
+               "d2h_bytes_per_step": down, "ms_per_step": t_e2e * 1e3}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline_lap25(A, c)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": gflops, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": CONFIGS[name][2], "stencil": name, "grid_per_gpu": list(ldims),
+                       "global_grid": list(gdims), "decomposition": f"z-slabs x{world}" if world > 1 else "none",
+                       "variant": info["variant"], "flops_per_point": flops_pt,
+                       "bytes_per_point": info["bytes_per_point"],
+                       "l2": "input 1 GiB/GPU > 126 MB L2 (no flush needed)"},
+            "hbm_gbs": total_pts * info["bytes_per_point"] * args.steps / (ms_max * 1e-3) / 1e9,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                         "kernel": "sdag_sweep<Lap25> " + info["variant"], "kernel_ms": kms},
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": clk.summary(),
+        }
+        print(json.dumps(line))
+    if dist:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,240 @@
+/*
+ * sdag.h -- C ABI of the B200-native FP64 stencil-DAG library ("sdag").
+ *
+ * Problem statement (Rawat et al., IPDPS 2019, /root/reference/PAPER.md,
+ * cited P:<line> <section>): a stencil computation "sweeps a computational
+ * grid, and updates the value at each point by reading a fixed neighborhood
+ * around it" (section I); the user declares arrays, scalars and
+ * iterators and writes the stencil function in a restricted C subset whose
+ * index expressions are iterator +- constant (section II); the
+ * declared arrays and scalars "will be passed as arguments to the generated
+ * host function" (Listing 1).  sdag plans such a DAG
+ * over N input and M output grids once (parse, analyse, choose a kernel
+ * variant) and applies it asynchronously on a CUDA stream.
+ *
+ * Conventions common to every entry point
+ * ---------------------------------------
+ *  - Status: every function returning sdag_status returns SDAG_OK (0) on
+ *    success.  On failure nothing has been enqueued, and sdag_last_error()
+ *    returns a thread-local message (parse errors carry "line:col").
+ *  - Grids: FP64, C order [nz][ny][nx] with x (iterator i, the innermost
+ *    iterator) contiguous; device pointers, 8-byte aligned
+ *    (16-byte aligned + nx even enables the TMA loader; otherwise the LSU
+ *    loader is used).  1D arrays are device pointers of the
+ *    length of the axis their iterator indexes.  Scalars are a HOST array of
+ *    doubles copied into kernel parameters at enqueue time.
+ *  - Argument order: 3D arrays, 1D arrays and scalars are each passed in the
+ *    order they appear among the stencil function's formal parameters
+ *    ("stencil jacobi (B, A, h2inv, a, b)"); sdag_plan_arg() reports
+ *    names and roles.
+ *  - Semantics (reading R1): out-of-place; only the interior
+ *    [R_a, n_a - R_a) of each axis a is written, R_a the maximal |offset|
+ *    read along a; every other element of every output is left
+ *    bit-identical.  An output may not alias an input (SDAG_ERR_INVALID_ARG).
+ *    "inout" arrays (read at offset 0 before being written, e.g. SW4's
+ *    uacc = a1*uacc + cof*r) are updated in place.
+ *  - Ownership: the caller owns all grid / 1D / scalar memory; a plan owns
+ *    only immutable metadata, a TMA-descriptor cache and (for
+ *    sdag_apply_host) a device workspace, all released by sdag_plan_destroy.
+ *  - Synchronicity: sdag_apply* enqueue on `stream` and never synchronise
+ *    (except sdag_apply_host, which is synchronous).  Device faults surface
+ *    at the caller's next synchronisation.
+ *  - No CPU fallback: a device that is not sm_100 returns SDAG_ERR_DEVICE.
+ */
+#ifndef SDAG_H
+#define SDAG_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SDAG_VERSION_MAJOR 0
+#define SDAG_VERSION_MINOR 1
+
+typedef enum sdag_status {
+    SDAG_OK = 0,
+    SDAG_ERR_INVALID_ARG = 1, /* null / wrong count / misaligned / aliasing / bad dims   */
+    SDAG_ERR_PARSE = 2,       /* spec text does not parse (message has line:col)          */
+    SDAG_ERR_SEMANTIC = 3,    /* parses but is ill-formed (undeclared name, bad index...) */
+    SDAG_ERR_UNSUPPORTED = 4, /* valid DAG outside the hot path (e.g. shifted writes)     */
+    SDAG_ERR_DOMAIN = 5,      /* dims too small for the radius, or order exceeded         */
+    SDAG_ERR_DEVICE = 6,      /* no CUDA device / not sm_100 / host-only plan applied     */
+    SDAG_ERR_CUDA = 7,        /* CUDA runtime / driver error (message has the CUDA text)  */
+    SDAG_ERR_NCCL = 8,        /* NCCL error or NCCL library not loadable                  */
+    SDAG_ERR_NOMEM = 9
+} sdag_status;
+
+typedef struct sdag_plan_s *sdag_plan;
+typedef struct sdag_dist_s *sdag_dist;
+typedef struct CUstream_st *sdag_stream; /* == cudaStream_t; NULL = legacy default stream */
+
+/* Device selector values for sdag_plan_opts.device */
+#define SDAG_DEVICE_CURRENT (-1)
+#define SDAG_DEVICE_NONE (-2) /* host-only plan: parse+analyse+plan, apply -> SDAG_ERR_DEVICE */
+
+typedef struct sdag_plan_opts {
+    int32_t order;             /* declared max radius (stencil order); -1 = infer.
+                                  Error SDAG_ERR_DOMAIN if any access exceeds it.          */
+    int32_t device;            /* CUDA ordinal, SDAG_DEVICE_CURRENT or SDAG_DEVICE_NONE    */
+    int32_t tune;              /* 0 = heuristic variant choice; 1 = time the candidates at
+                                  plan time on scratch buffers (hierarchical autotuning,
+                                  P:1202-1271) -- synchronises the device                  */
+    int32_t batch;             /* independent problems per apply (sdag_apply_batched); >= 1 */
+    const char *force_variant; /* NULL, or a variant name from sdag_plan_variant_name()    */
+} sdag_plan_opts;
+
+/* Fills `o` with the defaults {order=-1, device=CURRENT, tune=0, batch=1, NULL}. */
+void sdag_plan_opts_init(sdag_plan_opts *o);
+
+typedef struct sdag_plan_info {
+    int32_t n_arrays3d, n_arrays1d, n_scalars; /* formal parameters by kind           */
+    int32_t n_in, n_out, n_inout;              /* roles of the 3D arrays             */
+    int32_t n_statements, n_temporaries;
+    int32_t radius[3];                         /* z, y, x (per-axis order)            */
+    int64_t dims[3];                           /* nz, ny, nx                         */
+    int64_t lo[3], hi[3];                      /* interior [lo, hi) per axis          */
+    int64_t points;                            /* interior points per apply (1 problem) */
+    double flops_per_point;                    /* canonical count (R9)      */
+    double bytes_per_point;                    /* algorithmic HBM bytes / written pt   */
+    double oi_paper;                           /* flops / (8 * #IO arrays), Table III  */
+    int32_t n_kernels;                         /* launches per apply                   */
+    int32_t n_variants;                        /* candidate variants considered        */
+    const char *dag;                           /* registry DAG matched ("jacobi7", ...) */
+    const char *variant;                       /* chosen variant name                  */
+} sdag_plan_info;
+
+/*
+ * a1-a3: parse `spec` (the Listing-1 DSL, plus 1D arrays,
+ * #pragma and #assign, P:461-471 / P:513-533), analyse it (radius, roles,
+ * canonical flops/bytes; Table I) and choose a kernel
+ * variant for grids of `dims` = {nz, ny, nx} (for 1- or 2-iterator specs the
+ * missing leading extents must be 1).  `opts` may be NULL.  On success *out
+ * owns the plan.  Errors: PARSE, SEMANTIC, UNSUPPORTED, DOMAIN, DEVICE
+ * (device requested but unusable), INVALID_ARG.
+ */
+sdag_status sdag_plan_create(const char *spec, const int64_t dims[3], const sdag_plan_opts *opts,
+                             sdag_plan *out);
+sdag_status sdag_plan_info_get(sdag_plan plan, sdag_plan_info *out);
+/* kind: 0 = 3D array, 1 = 1D array, 2 = scalar; role (3D only): 0 in, 1 out, 2 inout.
+ * For 1D arrays *role is the axis (0 = z, 1 = y, 2 = x).  Strings live as long as the plan. */
+sdag_status sdag_plan_arg(sdag_plan plan, int32_t kind, int32_t idx, const char **name, int32_t *role);
+/* Candidate variants of this plan, 0 <= idx < info.n_variants. */
+sdag_status sdag_plan_variant_name(sdag_plan plan, int32_t idx, const char **name);
+/* Human-readable plan report (analysis counts, variant, launch geometry). */
+const char *sdag_plan_describe(sdag_plan plan);
+void sdag_plan_destroy(sdag_plan plan);
+
+/*
+ * a4-a5: one sweep.  arrays3d[n3d] device pointers (every 3D formal, in
+ * formal order, inputs and outputs alike), arrays1d[n1d] device pointers,
+ * scalars[nscalars] host doubles.  Enqueued on `stream`.
+ */
+sdag_status sdag_apply(sdag_plan plan, double *const *arrays3d, int32_t n3d, const double *const *arrays1d,
+                       int32_t n1d, const double *scalars, int32_t nscalars, sdag_stream stream);
+
+/* `batch` independent problems in ONE launch; every 3D array is [batch][nz][ny][nx]
+ * contiguous and every 1D array [batch][len].  batch <= opts.batch is not required. */
+sdag_status sdag_apply_batched(sdag_plan plan, int32_t batch, double *const *arrays3d, int32_t n3d,
+                               const double *const *arrays1d, int32_t n1d, const double *scalars,
+                               int32_t nscalars, sdag_stream stream);
+
+/*
+ * a6: T sweeps ping-pong (Fig 1a; time loop P:380-381) of a plan
+ * with exactly one 3D input and one 3D output (and no 1D arrays):
+ * sweep t reads buf[t&1] and writes the interior of buf[(t+1)&1].  Both
+ * buffers must hold identical boundary rings on entry (fixed Dirichlet
+ * ring).  Result in buf[T&1].
+ */
+sdag_status sdag_apply_iterated(sdag_plan plan, double *buf0, double *buf1, int32_t T, const double *scalars,
+                                int32_t nscalars, sdag_stream stream);
+
+/*
+ * End-to-end call with HOST buffers (pageable or pinned): copies every 3D
+ * input/inout and 1D array host->device into a plan-owned workspace, runs
+ * one sweep, copies every output/inout device->host, and synchronises
+ * `stream`.  h2d_bytes / d2h_bytes (nullable) receive the bytes moved.
+ */
+sdag_status sdag_apply_host(sdag_plan plan, double *const *host3d, int32_t n3d, const double *const *host1d,
+                            int32_t n1d, const double *scalars, int32_t nscalars, sdag_stream stream,
+                            int64_t *h2d_bytes, int64_t *d2h_bytes);
+
+/* ------------------------------------------------------------------------
+ * a7: z-slab domain decomposition with per-sweep halo exchange
+ * (north-star addition; the paper is single-GPU).
+ * Rank p owns global interior-capable planes [z0_p, z0_p + nz_p); its local
+ * allocation is (R_z + nz_p + R_z) planes: R_z ghost planes below and above.
+ * ------------------------------------------------------------------------ */
+
+/* Pure host logic, no device: partition of `global_nz` planes over `nranks`
+ * for radius `rz`.  out[0] = first owned global plane, out[1] = owned planes,
+ * out[2] = local allocation planes (owned + 2 rz), out[3] = first local plane
+ * this rank computes, out[4] = one past the last, out[5] = 1 if the rank has
+ * a lower neighbour, out[6] = 1 if it has an upper neighbour.  Remainder
+ * planes go to the lowest ranks.  Error DOMAIN if some rank would own < rz. */
+sdag_status sdag_slab_partition(int64_t global_nz, int32_t rz, int32_t nranks, int32_t rank, int64_t out[7]);
+
+/* Pure host logic: the per-sweep halo schedule of that rank, in LOCAL plane
+ * indices (rz planes each).  out[0] = first plane sent to the lower
+ * neighbour, out[1] = first ghost plane received from it, out[2] / out[3] the
+ * same for the upper neighbour (-1 = no such neighbour), out[4] = rz. */
+sdag_status sdag_slab_halo(int64_t global_nz, int32_t rz, int32_t nranks, int32_t rank, int64_t out[5]);
+
+/* NCCL bootstrap through the same libnccl.so.2 torch loads (dlopen).
+ * unique id: 128 bytes, broadcast by the caller (e.g. torch.distributed). */
+sdag_status sdag_nccl_get_unique_id(uint8_t id[128]);
+sdag_status sdag_nccl_comm_create(const uint8_t id[128], int32_t nranks, int32_t rank, int32_t device,
+                                  void **comm);
+void sdag_nccl_comm_destroy(void *comm);
+
+/* Create this rank's slab of a `global_dims` problem.  `nccl_comm` is an
+ * ncclComm_t from sdag_nccl_comm_create (or NULL when nranks == 1). */
+sdag_status sdag_dist_create(const char *spec, const int64_t global_dims[3], const sdag_plan_opts *opts,
+                             int32_t rank, int32_t nranks, void *nccl_comm, sdag_dist *out);
+/* local_dims = {nz_alloc, ny, nx}; global_z_of_local0 = global plane index of local plane 0 */
+sdag_status sdag_dist_layout(sdag_dist d, int64_t local_dims[3], int64_t *global_z_of_local0);
+sdag_plan sdag_dist_local_plan(sdag_dist d);
+
+/* One sweep of a slab: exchange the R_z boundary planes of every z-staged
+ * input with the neighbours (NCCL send/recv on `comm`, or an internal stream
+ * if NULL), compute owned planes that need no ghosts on `compute`
+ * concurrently, then the ghost-dependent planes.  1D z-arrays span the local
+ * allocation.  Ordered on `compute` on return. */
+sdag_status sdag_dist_apply(sdag_dist d, double *const *arrays3d, int32_t n3d, const double *const *arrays1d,
+                            int32_t n1d, const double *scalars, int32_t nscalars, sdag_stream compute,
+                            sdag_stream comm);
+/* T sweeps, ping-pong, exchange every sweep (1 in -> 1 out plans). Result in buf[T&1]. */
+sdag_status sdag_dist_apply_iterated(sdag_dist d, double *buf0, double *buf1, int32_t T, const double *scalars,
+                                     int32_t nscalars, sdag_stream compute, sdag_stream comm);
+void sdag_dist_destroy(sdag_dist d);
+
+/* Loopback exchanger (all slabs in one process on one device; halos moved
+ * with cudaMemcpyAsync): same index bookkeeping as the NCCL path, for
+ * bit-exact single-GPU tests.  dists[r] from sdag_dist_create(..., r, n, NULL). */
+sdag_status sdag_dist_apply_iterated_loopback(sdag_dist *dists, int32_t nranks, double *const *buf0,
+                                              double *const *buf1, int32_t T, const double *scalars,
+                                              int32_t nscalars, sdag_stream stream);
+
+/* ------------------------------------------------------------------------
+ * Diagnostics
+ * ------------------------------------------------------------------------ */
+const char *sdag_last_error(void); /* thread-local; valid until the next sdag_* call on this thread */
+const char *sdag_version(void);
+/* Number of sweep-kernel launches this process has enqueued (all plans). */
+int64_t sdag_launch_count(void);
+/* FP64 peak micro-benchmark (dependent-chain-free DFMA over all SMs) on the
+ * current device; returns achieved FLOP/s in *flops (synchronous). */
+sdag_status sdag_measure_fp64_peak(double *flops, sdag_stream stream);
+
+/* Registered DAGs with hand-written sm_100a bodies: name and canonical spec
+ * text (a spec whose canonical form equals one of these, up to renaming, is
+ * accepted by sdag_plan_create).  Strings live for the process. */
+int32_t sdag_registry_count(void);
+sdag_status sdag_registry_get(int32_t idx, const char **name, const char **text);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SDAG_H */

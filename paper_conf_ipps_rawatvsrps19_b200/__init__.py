@@ -1,0 +1,308 @@
+"""sdag -- B200-native FP64 stencil-DAG library (Python binding).
+
+Thin marshalling layer over the C ABI in include/sdag.h (libsdag.so): every
+step of the hot path -- parse (a1), analyse (a2), plan (a3), the sm_100a
+sweep kernels (a4-a6) and the z-slab halo exchange (a7) -- runs in the native
+library.  PyTorch is used only to own device memory and streams.
+
+    import paper_conf_ipps_rawatvsrps19_b200 as sdag
+    plan = sdag.Plan(sdag.spec_text("lap25"), (512, 512, 512))
+    plan.apply([out, inp], scalars=[c0, c1, c2, c3, c4])   # formal order (B, A, c0..c4)
+
+Reference: Rawat et al., "On Optimizing Complex Stencils on GPUs", IPDPS 2019
+(PAPER.md): Listing 1 DSL, streaming, Table I
+benchmarks.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+from . import _capi
+from ._capi import PlanInfo, PlanOpts, SDAG_DEVICE_CURRENT, SDAG_DEVICE_NONE
+
+__all__ = ["Plan", "Dist", "SdagError", "registry", "spec_text", "slab_partition", "slab_halo", "nccl_unique_id",
+           "nccl_comm_create", "nccl_comm_destroy", "launch_count", "fp64_peak", "version", "SPEC_DIR"]
+
+SPEC_DIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "specs")
+
+
+class SdagError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"sdag {_capi.STATUS.get(status, status)}: {msg}")
+        self.status = status
+        self.code = _capi.STATUS.get(status, str(status))
+
+
+def _check(st: int):
+    if st != 0:
+        raise SdagError(st, (_capi.lib().sdag_last_error() or b"").decode())
+
+
+def _stream_handle(stream):
+    if stream is None:
+        import torch
+        return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, int):
+        return ctypes.c_void_p(stream)
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _ptr(t, what):
+    """device pointer of a contiguous float64 CUDA tensor (no copies)"""
+    import torch
+    if not isinstance(t, torch.Tensor):
+        raise TypeError(f"{what}: expected a torch.Tensor")
+    if t.dtype != torch.float64 or not t.is_cuda or not t.is_contiguous():
+        raise TypeError(f"{what}: need a contiguous float64 CUDA tensor (got {t.dtype}, {t.device})")
+    return t.data_ptr()
+
+
+def _arr(ptrs):
+    return (ctypes.c_void_p * max(1, len(ptrs)))(*ptrs)
+
+
+def _scal(s):
+    s = [float(x) for x in (s or [])]
+    return (ctypes.c_double * max(1, len(s)))(*s), len(s)
+
+
+def _opts(order=-1, device=None, tune=False, batch=1, variant=None):
+    o = PlanOpts()
+    _capi.lib().sdag_plan_opts_init(ctypes.byref(o))
+    o.order = int(order)
+    if device == "none":
+        o.device = SDAG_DEVICE_NONE
+    elif device is None:
+        o.device = SDAG_DEVICE_CURRENT
+    else:
+        o.device = int(device)
+    o.tune = 1 if tune else 0
+    o.batch = int(batch)
+    o.force_variant = variant.encode() if variant else None
+    return o
+
+
+def registry() -> dict:
+    """Registered DAGs with hand-written sm_100a bodies: name -> canonical spec text."""
+    L = _capi.lib()
+    out = {}
+    for i in range(L.sdag_registry_count()):
+        n, t = ctypes.c_char_p(), ctypes.c_char_p()
+        _check(L.sdag_registry_get(i, ctypes.byref(n), ctypes.byref(t)))
+        out[n.value.decode()] = t.value.decode()
+    return out
+
+
+def spec_text(name: str) -> str:
+    with open(os.path.join(SPEC_DIR, name + ".sdag")) as f:
+        return f.read()
+
+
+class Plan:
+    """A planned stencil DAG (a1-a3) bound to grid dims (nz, ny, nx)."""
+
+    def __init__(self, spec: str, dims, order=-1, device=None, tune=False, batch=1, variant=None):
+        self._L = _capi.lib()
+        self._h = ctypes.c_void_p()
+        d = (ctypes.c_int64 * 3)(*[int(x) for x in dims])
+        o = _opts(order, device, tune, batch, variant)
+        _check(self._L.sdag_plan_create(spec.encode(), d, ctypes.byref(o), ctypes.byref(self._h)))
+        self._owned = True
+
+    @classmethod
+    def _borrow(cls, handle):
+        p = cls.__new__(cls)
+        p._L = _capi.lib()
+        p._h = ctypes.c_void_p(handle)
+        p._owned = False
+        return p
+
+    def close(self):
+        if getattr(self, "_owned", False) and self._h:
+            self._L.sdag_plan_destroy(self._h)
+        self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    # ---- introspection ----
+    @property
+    def info(self) -> dict:
+        i = PlanInfo()
+        _check(self._L.sdag_plan_info_get(self._h, ctypes.byref(i)))
+        d = {f: getattr(i, f) for f, _ in PlanInfo._fields_}
+        for k in ("radius", "dims", "lo", "hi"):
+            d[k] = tuple(d[k])
+        d["dag"] = i.dag.decode()
+        d["variant"] = i.variant.decode()
+        return d
+
+    def args(self):
+        """[(kind, index, name, role_or_axis)] in formal order per kind."""
+        i = self.info
+        out = []
+        for kind, n in ((0, i["n_arrays3d"]), (1, i["n_arrays1d"]), (2, i["n_scalars"])):
+            for q in range(n):
+                nm, r = ctypes.c_char_p(), ctypes.c_int32()
+                _check(self._L.sdag_plan_arg(self._h, kind, q, ctypes.byref(nm), ctypes.byref(r)))
+                out.append((kind, q, nm.value.decode(), r.value))
+        return out
+
+    def arg_names(self, kind: int):
+        return [a[2] for a in self.args() if a[0] == kind]
+
+    def variants(self):
+        out = []
+        for q in range(self.info["n_variants"]):
+            nm = ctypes.c_char_p()
+            _check(self._L.sdag_plan_variant_name(self._h, q, ctypes.byref(nm)))
+            out.append(nm.value.decode())
+        return out
+
+    def describe(self) -> str:
+        return self._L.sdag_plan_describe(self._h).decode()
+
+    # ---- apply ----
+    def apply(self, arrays3d, arrays1d=(), scalars=(), stream=None):
+        p3 = [_ptr(t, "grid array") for t in arrays3d]
+        p1 = [_ptr(t, "1D array") for t in arrays1d]
+        s, ns = _scal(scalars)
+        _check(self._L.sdag_apply(self._h, _arr(p3), len(p3), _arr(p1), len(p1), s, ns, _stream_handle(stream)))
+
+    def apply_batched(self, batch, arrays3d, arrays1d=(), scalars=(), stream=None):
+        p3 = [_ptr(t, "grid array") for t in arrays3d]
+        p1 = [_ptr(t, "1D array") for t in arrays1d]
+        s, ns = _scal(scalars)
+        _check(self._L.sdag_apply_batched(self._h, int(batch), _arr(p3), len(p3), _arr(p1), len(p1), s, ns,
+                                          _stream_handle(stream)))
+
+    def apply_iterated(self, buf0, buf1, T, scalars=(), stream=None):
+        s, ns = _scal(scalars)
+        _check(self._L.sdag_apply_iterated(self._h, _ptr(buf0, "buf0"), _ptr(buf1, "buf1"), int(T), s, ns,
+                                           _stream_handle(stream)))
+
+    def apply_host(self, host3d, host1d=(), scalars=(), stream=None):
+        """End-to-end call with host numpy buffers (outputs/inouts updated in place).
+        Returns (h2d_bytes, d2h_bytes)."""
+        import numpy as np
+        for a in list(host3d) + list(host1d):
+            if not (isinstance(a, np.ndarray) and a.dtype == np.float64 and a.flags.c_contiguous):
+                raise TypeError("apply_host needs contiguous float64 numpy arrays")
+        p3 = [a.ctypes.data for a in host3d]
+        p1 = [a.ctypes.data for a in host1d]
+        s, ns = _scal(scalars)
+        up, down = ctypes.c_int64(), ctypes.c_int64()
+        _check(self._L.sdag_apply_host(self._h, _arr(p3), len(p3), _arr(p1), len(p1), s, ns, _stream_handle(stream),
+                                       ctypes.byref(up), ctypes.byref(down)))
+        return up.value, down.value
+
+
+def slab_partition(global_nz: int, rz: int, nranks: int, rank: int) -> dict:
+    out = (ctypes.c_int64 * 7)()
+    _check(_capi.lib().sdag_slab_partition(int(global_nz), int(rz), int(nranks), int(rank), out))
+    keys = ("z0", "nz_own", "nz_alloc", "k_lo", "k_hi", "has_lower", "has_upper")
+    return dict(zip(keys, list(out)))
+
+
+def slab_halo(global_nz: int, rz: int, nranks: int, rank: int) -> dict:
+    out = (ctypes.c_int64 * 5)()
+    _check(_capi.lib().sdag_slab_halo(int(global_nz), int(rz), int(nranks), int(rank), out))
+    return dict(zip(("lo_send", "lo_recv", "up_send", "up_recv", "planes"), list(out)))
+
+
+def nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(_capi.lib().sdag_nccl_get_unique_id(buf))
+    return buf.raw
+
+
+def nccl_comm_create(uid: bytes, nranks: int, rank: int, device: int) -> int:
+    c = ctypes.c_void_p()
+    _check(_capi.lib().sdag_nccl_comm_create(uid, int(nranks), int(rank), int(device), ctypes.byref(c)))
+    return c.value
+
+
+def nccl_comm_destroy(comm: int):
+    _capi.lib().sdag_nccl_comm_destroy(ctypes.c_void_p(comm))
+
+
+class Dist:
+    """This rank's z-slab of a global stencil problem (a7)."""
+
+    def __init__(self, spec, global_dims, rank, nranks, comm=None, order=-1, device=None, tune=False, variant=None):
+        self._L = _capi.lib()
+        self._h = ctypes.c_void_p()
+        d = (ctypes.c_int64 * 3)(*[int(x) for x in global_dims])
+        o = _opts(order, device, tune, 1, variant)
+        _check(self._L.sdag_dist_create(spec.encode(), d, ctypes.byref(o), int(rank), int(nranks),
+                                        ctypes.c_void_p(comm or 0), ctypes.byref(self._h)))
+        self.rank, self.nranks = rank, nranks
+
+    def close(self):
+        if self._h:
+            self._L.sdag_dist_destroy(self._h)
+        self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def layout(self):
+        """(local_dims (nz_alloc, ny, nx), global z of local plane 0)"""
+        ld = (ctypes.c_int64 * 3)()
+        g = ctypes.c_int64()
+        _check(self._L.sdag_dist_layout(self._h, ld, ctypes.byref(g)))
+        return tuple(ld), g.value
+
+    @property
+    def plan(self) -> Plan:
+        return Plan._borrow(self._L.sdag_dist_local_plan(self._h))
+
+    def apply(self, arrays3d, arrays1d=(), scalars=(), stream=None, comm_stream=None):
+        p3 = [_ptr(t, "grid array") for t in arrays3d]
+        p1 = [_ptr(t, "1D array") for t in arrays1d]
+        s, ns = _scal(scalars)
+        cs = ctypes.c_void_p(0) if comm_stream is None else _stream_handle(comm_stream)
+        _check(self._L.sdag_dist_apply(self._h, _arr(p3), len(p3), _arr(p1), len(p1), s, ns, _stream_handle(stream),
+                                       cs))
+
+    def apply_iterated(self, buf0, buf1, T, scalars=(), stream=None, comm_stream=None):
+        s, ns = _scal(scalars)
+        cs = ctypes.c_void_p(0) if comm_stream is None else _stream_handle(comm_stream)
+        _check(self._L.sdag_dist_apply_iterated(self._h, _ptr(buf0, "buf0"), _ptr(buf1, "buf1"), int(T), s, ns,
+                                                _stream_handle(stream), cs))
+
+    @staticmethod
+    def apply_iterated_loopback(dists, bufs0, bufs1, T, scalars=(), stream=None):
+        hs = (ctypes.c_void_p * len(dists))(*[d._h.value for d in dists])
+        b0 = _arr([_ptr(t, "buf0") for t in bufs0])
+        b1 = _arr([_ptr(t, "buf1") for t in bufs1])
+        s, ns = _scal(scalars)
+        _check(_capi.lib().sdag_dist_apply_iterated_loopback(hs, len(dists), b0, b1, int(T), s, ns,
+                                                            _stream_handle(stream)))
+
+
+def launch_count() -> int:
+    return int(_capi.lib().sdag_launch_count())
+
+
+def fp64_peak(stream=None) -> float:
+    f = ctypes.c_double()
+    _check(_capi.lib().sdag_measure_fp64_peak(ctypes.byref(f), _stream_handle(stream)))
+    return f.value
+
+
+def version() -> str:
+    return _capi.lib().sdag_version().decode()

@@ -1,0 +1,244 @@
+// capi.cpp -- the extern "C" boundary (include/sdag.h): argument checks,
+// exception -> sdag_status translation, thread-local error text.
+#include <cuda_runtime.h>
+
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "dist.hpp"
+#include "plan.hpp"
+#include "sdag.h"
+
+namespace {
+
+thread_local std::string g_err;
+
+template <class F>
+sdag_status guard(F &&f) {
+    g_err.clear();
+    try {
+        f();
+        return SDAG_OK;
+    } catch (const sdag::Error &e) {
+        g_err = e.what();
+        return static_cast<sdag_status>(e.status);
+    } catch (const std::bad_alloc &) {
+        g_err = "out of host memory";
+        return SDAG_ERR_NOMEM;
+    } catch (const std::exception &e) {
+        g_err = std::string("internal error: ") + e.what();
+        return SDAG_ERR_INVALID_ARG;
+    }
+}
+
+sdag::Plan *P(sdag_plan p) {
+    if (!p || !p->p) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null plan");
+    return p->p;
+}
+
+}  // namespace
+
+extern "C" {
+
+void sdag_plan_opts_init(sdag_plan_opts *o) {
+    if (!o) return;
+    o->order = -1;
+    o->device = SDAG_DEVICE_CURRENT;
+    o->tune = 0;
+    o->batch = 1;
+    o->force_variant = nullptr;
+}
+
+sdag_status sdag_plan_create(const char *spec, const int64_t dims[3], const sdag_plan_opts *opts, sdag_plan *out) {
+    return guard([&] {
+        if (!spec || !dims || !out) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null argument");
+        *out = nullptr;
+        sdag_plan_opts o;
+        sdag_plan_opts_init(&o);
+        if (opts) o = *opts;
+        sdag::Plan *p = sdag::plan_create(spec, dims, o);
+        *out = new sdag_plan_s{p};
+    });
+}
+
+sdag_status sdag_plan_info_get(sdag_plan plan, sdag_plan_info *out) {
+    return guard([&] {
+        if (!out) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null info");
+        sdag::plan_fill_info(P(plan), out);
+    });
+}
+
+sdag_status sdag_plan_arg(sdag_plan plan, int32_t kind, int32_t idx, const char **name, int32_t *role) {
+    return guard([&] {
+        sdag::Plan *p = P(plan);
+        if (kind < 0 || kind > 2) throw sdag::Error(SDAG_ERR_INVALID_ARG, "kind must be 0, 1 or 2");
+        const auto k = static_cast<sdag::ArgKind>(kind);
+        if (idx < 0 || idx >= p->st.n_of(k)) throw sdag::Error(SDAG_ERR_INVALID_ARG, "index out of range");
+        const sdag::Formal &f = p->st.formal(k, idx);
+        if (name) *name = f.name.c_str();
+        if (role) *role = (k == sdag::ArgKind::Array3D) ? int32_t(f.role) : (k == sdag::ArgKind::Array1D ? f.axis : -1);
+    });
+}
+
+sdag_status sdag_plan_variant_name(sdag_plan plan, int32_t idx, const char **name) {
+    return guard([&] {
+        sdag::Plan *p = P(plan);
+        if (idx < 0 || idx >= int(p->cands.size())) throw sdag::Error(SDAG_ERR_INVALID_ARG, "index out of range");
+        if (name) *name = p->cands[idx]->variant.c_str();
+    });
+}
+
+const char *sdag_plan_describe(sdag_plan plan) {
+    if (!plan || !plan->p) return "";
+    return plan->p->describe_text.c_str();
+}
+
+void sdag_plan_destroy(sdag_plan plan) {
+    if (!plan) return;
+    delete plan->p;
+    delete plan;
+}
+
+sdag_status sdag_apply(sdag_plan plan, double *const *a3, int32_t n3, const double *const *a1, int32_t n1,
+                       const double *s, int32_t ns, sdag_stream stream) {
+    return guard([&] { sdag::apply(P(plan), a3, n3, a1, n1, s, ns, 1, reinterpret_cast<cudaStream_t>(stream)); });
+}
+
+sdag_status sdag_apply_batched(sdag_plan plan, int32_t batch, double *const *a3, int32_t n3,
+                               const double *const *a1, int32_t n1, const double *s, int32_t ns,
+                               sdag_stream stream) {
+    return guard(
+        [&] { sdag::apply(P(plan), a3, n3, a1, n1, s, ns, batch, reinterpret_cast<cudaStream_t>(stream)); });
+}
+
+sdag_status sdag_apply_iterated(sdag_plan plan, double *b0, double *b1, int32_t T, const double *s, int32_t ns,
+                                sdag_stream stream) {
+    return guard(
+        [&] { sdag::apply_iterated(P(plan), b0, b1, T, s, ns, reinterpret_cast<cudaStream_t>(stream)); });
+}
+
+sdag_status sdag_apply_host(sdag_plan plan, double *const *h3, int32_t n3, const double *const *h1, int32_t n1,
+                            const double *s, int32_t ns, sdag_stream stream, int64_t *h2d, int64_t *d2h) {
+    return guard([&] {
+        sdag::apply_host(P(plan), h3, n3, h1, n1, s, ns, reinterpret_cast<cudaStream_t>(stream), h2d, d2h);
+    });
+}
+
+// ---- distributed ------------------------------------------------------------
+
+sdag_status sdag_slab_partition(int64_t global_nz, int32_t rz, int32_t nranks, int32_t rank, int64_t out[7]) {
+    return guard([&] {
+        if (!out) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null out");
+        sdag::Slab s = sdag::slab_partition(global_nz, rz, nranks, rank);
+        out[0] = s.z0;
+        out[1] = s.nz_own;
+        out[2] = s.nz_alloc;
+        out[3] = s.k_lo;
+        out[4] = s.k_hi;
+        out[5] = s.has_lower;
+        out[6] = s.has_upper;
+    });
+}
+
+sdag_status sdag_slab_halo(int64_t global_nz, int32_t rz, int32_t nranks, int32_t rank, int64_t out[5]) {
+    return guard([&] {
+        if (!out) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null out");
+        sdag::Halo h = sdag::halo_schedule(sdag::slab_partition(global_nz, rz, nranks, rank), rz);
+        out[0] = h.lo_send;
+        out[1] = h.lo_recv;
+        out[2] = h.up_send;
+        out[3] = h.up_recv;
+        out[4] = h.planes;
+    });
+}
+
+sdag_status sdag_nccl_get_unique_id(uint8_t id[128]) {
+    return guard([&] { sdag::nccl_unique_id(id); });
+}
+
+sdag_status sdag_nccl_comm_create(const uint8_t id[128], int32_t nranks, int32_t rank, int32_t device, void **comm) {
+    return guard([&] { *comm = sdag::nccl_comm_create(id, nranks, rank, device); });
+}
+
+void sdag_nccl_comm_destroy(void *comm) { sdag::nccl_comm_destroy(comm); }
+
+sdag_status sdag_dist_create(const char *spec, const int64_t global_dims[3], const sdag_plan_opts *opts,
+                             int32_t rank, int32_t nranks, void *nccl_comm, sdag_dist *out) {
+    return guard([&] {
+        if (!spec || !global_dims || !out) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null argument");
+        sdag_plan_opts o;
+        sdag_plan_opts_init(&o);
+        if (opts) o = *opts;
+        *out = reinterpret_cast<sdag_dist>(sdag::dist_create(spec, global_dims, o, rank, nranks, nccl_comm));
+    });
+}
+
+sdag_status sdag_dist_layout(sdag_dist d, int64_t local_dims[3], int64_t *gz0) {
+    return guard([&] {
+        auto *D = reinterpret_cast<sdag::Dist *>(d);
+        if (!D) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null dist");
+        for (int a = 0; a < 3; a++) local_dims[a] = D->local->dims[a];
+        if (gz0) *gz0 = D->slab.z0 - D->rz;
+    });
+}
+
+sdag_plan sdag_dist_local_plan(sdag_dist d) {
+    auto *D = reinterpret_cast<sdag::Dist *>(d);
+    return D ? reinterpret_cast<sdag_plan>(&D->handle) : nullptr;
+}
+
+sdag_status sdag_dist_apply(sdag_dist d, double *const *a3, int32_t n3, const double *const *a1, int32_t n1,
+                            const double *s, int32_t ns, sdag_stream compute, sdag_stream comm) {
+    return guard([&] {
+        sdag::dist_apply(reinterpret_cast<sdag::Dist *>(d), a3, n3, a1, n1, s, ns,
+                         reinterpret_cast<cudaStream_t>(compute), reinterpret_cast<cudaStream_t>(comm));
+    });
+}
+
+sdag_status sdag_dist_apply_iterated(sdag_dist d, double *b0, double *b1, int32_t T, const double *s, int32_t ns,
+                                     sdag_stream compute, sdag_stream comm) {
+    return guard([&] {
+        sdag::dist_apply_iterated(reinterpret_cast<sdag::Dist *>(d), b0, b1, T, s, ns,
+                                  reinterpret_cast<cudaStream_t>(compute), reinterpret_cast<cudaStream_t>(comm));
+    });
+}
+
+sdag_status sdag_dist_apply_iterated_loopback(sdag_dist *dists, int32_t nranks, double *const *b0,
+                                              double *const *b1, int32_t T, const double *s, int32_t ns,
+                                              sdag_stream stream) {
+    return guard([&] {
+        sdag::dist_apply_iterated_loopback(reinterpret_cast<sdag::Dist **>(dists), nranks, b0, b1, T, s, ns,
+                                           reinterpret_cast<cudaStream_t>(stream));
+    });
+}
+
+void sdag_dist_destroy(sdag_dist d) { delete reinterpret_cast<sdag::Dist *>(d); }
+
+// ---- diagnostics ------------------------------------------------------------
+
+const char *sdag_last_error(void) { return g_err.c_str(); }
+
+const char *sdag_version(void) { return "sdag 0.1 (sm_100a)"; }
+
+int64_t sdag_launch_count(void) { return sdag::launch_count(); }
+
+sdag_status sdag_measure_fp64_peak(double *flops, sdag_stream stream) {
+    return guard([&] {
+        if (!flops) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null out");
+        *flops = sdag::measure_fp64_peak(reinterpret_cast<cudaStream_t>(stream));
+    });
+}
+
+int32_t sdag_registry_count(void) { return int32_t(sdag::registry().size()); }
+
+sdag_status sdag_registry_get(int32_t idx, const char **name, const char **text) {
+    return guard([&] {
+        const auto &r = sdag::registry();
+        if (idx < 0 || idx >= int(r.size())) throw sdag::Error(SDAG_ERR_INVALID_ARG, "index out of range");
+        if (name) *name = r[idx].name.c_str();
+        if (text) *text = r[idx].text.c_str();
+    });
+}
+
+}  // extern "C"

@@ -1,0 +1,358 @@
+// dist.cpp -- a7: z-slab decomposition (north-star addition; the paper is
+// single-GPU).  Rank p owns a contiguous range of global z-planes;
+// its local allocation adds R_z ghost planes below and above.  Every sweep:
+//   comm stream:    ncclGroupStart; send my R_z lowest/highest owned planes of
+//                   each z-read input to rank-1/rank+1; recv their planes into
+//                   my ghosts; ncclGroupEnd              (no packing: C-order
+//                   z-planes are contiguous)
+//   compute stream: concurrently, the sweep kernel over owned planes that read
+//                   no ghost; then (event join) the same kernel over the
+//                   R_z planes next to each ghost layer.
+// Interior and boundary launches run the same kernel instantiation, so the
+// result is bit-identical to a single-GPU sweep of the global grid.
+#include "dist.hpp"
+
+#include <dlfcn.h>
+
+#include <cstdlib>
+#include <cstring>
+
+#include "sdag.h"
+
+namespace sdag {
+
+// ---------------------------------------------------------------------------
+// host logic
+// ---------------------------------------------------------------------------
+
+Slab slab_partition(int64_t gnz, int rz, int nranks, int rank) {
+    if (nranks < 1 || rank < 0 || rank >= nranks) throw Error(SDAG_ERR_INVALID_ARG, "bad rank / nranks");
+    if (rz < 0) throw Error(SDAG_ERR_INVALID_ARG, "negative radius");
+    if (gnz < 2 * int64_t(rz) + 1) throw Error(SDAG_ERR_DOMAIN, "global z extent has no interior");
+    Slab s;
+    const int64_t base = gnz / nranks, rem = gnz % nranks;
+    s.nz_own = base + (rank < rem ? 1 : 0);
+    s.z0 = int64_t(rank) * base + std::min<int64_t>(rank, rem);
+    if (base < std::max(rz, 1))
+        throw Error(SDAG_ERR_DOMAIN, "every rank must own at least max(R_z,1) = " + std::to_string(std::max(rz, 1)) +
+                                         " planes (global nz " + std::to_string(gnz) + ", " +
+                                         std::to_string(nranks) + " ranks)");
+    s.nz_alloc = s.nz_own + 2 * rz;
+    const int64_t g_of_l0 = s.z0 - rz;  // global plane of local plane 0
+    const int64_t glo = std::max<int64_t>(s.z0, rz), ghi = std::min<int64_t>(s.z0 + s.nz_own, gnz - rz);
+    s.k_lo = glo - g_of_l0;
+    s.k_hi = std::max(ghi - g_of_l0, s.k_lo);
+    s.has_lower = rank > 0;
+    s.has_upper = rank < nranks - 1;
+    return s;
+}
+
+Halo halo_schedule(const Slab &s, int rz) {
+    Halo h;
+    h.planes = rz;
+    if (rz == 0) return h;
+    if (s.has_lower) {
+        h.lo_send = rz;  // my lowest rz owned planes
+        h.lo_recv = 0;   // ghosts below
+    }
+    if (s.has_upper) {
+        h.up_send = s.nz_alloc - 2 * rz;  // my highest rz owned planes
+        h.up_recv = s.nz_alloc - rz;      // ghosts above
+    }
+    return h;
+}
+
+// ---------------------------------------------------------------------------
+// NCCL, loaded from the libnccl.so.2 the process already uses (torch's)
+// ---------------------------------------------------------------------------
+
+namespace {
+
+typedef int ncclResult_t;
+typedef struct ncclComm *ncclComm_t;
+struct ncclUniqueId {
+    char internal[128];
+};
+constexpr int ncclFloat64 = 8;
+
+struct NcclApi {
+    ncclResult_t (*GetUniqueId)(ncclUniqueId *) = nullptr;
+    ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*Send)(const void *, size_t, int, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*Recv)(void *, size_t, int, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*GroupStart)() = nullptr;
+    ncclResult_t (*GroupEnd)() = nullptr;
+    const char *(*GetErrorString)(ncclResult_t) = nullptr;
+    std::string err;
+};
+
+const NcclApi &nccl() {
+    static NcclApi a = [] {
+        NcclApi x;
+        const char *cands[] = {std::getenv("SDAG_NCCL_LIB"), "libnccl.so.2", "libnccl.so"};
+        void *h = nullptr;
+        for (const char *c : cands)
+            if (c && (h = dlopen(c, RTLD_NOW | RTLD_GLOBAL))) break;
+        if (!h) {
+            x.err = "cannot dlopen libnccl.so.2 (import torch first, or set SDAG_NCCL_LIB)";
+            return x;
+        }
+        auto sym = [&](const char *n) { return dlsym(h, n); };
+        x.GetUniqueId = reinterpret_cast<decltype(x.GetUniqueId)>(sym("ncclGetUniqueId"));
+        x.CommInitRank = reinterpret_cast<decltype(x.CommInitRank)>(sym("ncclCommInitRank"));
+        x.CommDestroy = reinterpret_cast<decltype(x.CommDestroy)>(sym("ncclCommDestroy"));
+        x.Send = reinterpret_cast<decltype(x.Send)>(sym("ncclSend"));
+        x.Recv = reinterpret_cast<decltype(x.Recv)>(sym("ncclRecv"));
+        x.GroupStart = reinterpret_cast<decltype(x.GroupStart)>(sym("ncclGroupStart"));
+        x.GroupEnd = reinterpret_cast<decltype(x.GroupEnd)>(sym("ncclGroupEnd"));
+        x.GetErrorString = reinterpret_cast<decltype(x.GetErrorString)>(sym("ncclGetErrorString"));
+        if (!x.GetUniqueId || !x.CommInitRank || !x.Send || !x.Recv || !x.GroupStart || !x.GroupEnd)
+            x.err = "libnccl.so.2 lacks the point-to-point API";
+        return x;
+    }();
+    if (!a.err.empty()) throw Error(SDAG_ERR_NCCL, a.err);
+    return a;
+}
+
+void nck(ncclResult_t r, const char *what) {
+    if (r != 0) {
+        const NcclApi &a = nccl();
+        throw Error(SDAG_ERR_NCCL, std::string(what) + ": " + (a.GetErrorString ? a.GetErrorString(r) : "error"));
+    }
+}
+
+}  // namespace
+
+void nccl_unique_id(uint8_t id[128]) {
+    ncclUniqueId u;
+    nck(nccl().GetUniqueId(&u), "ncclGetUniqueId");
+    std::memcpy(id, u.internal, 128);
+}
+
+void *nccl_comm_create(const uint8_t id[128], int nranks, int rank, int device) {
+    ncclUniqueId u;
+    std::memcpy(u.internal, id, 128);
+    if (device >= 0) check_cuda(cudaSetDevice(device), "cudaSetDevice");
+    ncclComm_t c = nullptr;
+    nck(nccl().CommInitRank(&c, nranks, u, rank), "ncclCommInitRank");
+    return c;
+}
+
+void nccl_comm_destroy(void *c) {
+    if (c) {
+        try {
+            nccl().CommDestroy(static_cast<ncclComm_t>(c));
+        } catch (...) {
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// dist plan
+// ---------------------------------------------------------------------------
+
+Dist::~Dist() {
+    if (own_comm) cudaStreamDestroy(own_comm);
+    if (ev_ready) cudaEventDestroy(ev_ready);
+    if (ev_halo) cudaEventDestroy(ev_halo);
+    delete local;
+}
+
+Dist *dist_create(const std::string &spec, const int64_t gdims[3], const sdag_plan_opts &o, int rank, int nranks,
+                  void *comm) {
+    if (nranks > 1 && !comm && o.device != SDAG_DEVICE_NONE) {
+        // allowed: loopback use (dist_apply_iterated_loopback); NCCL entry points check comm
+    }
+    // analyse once on the global grid to get R_z (host-only)
+    sdag_plan_opts ho = o;
+    ho.device = SDAG_DEVICE_NONE;
+    ho.tune = 0;
+    std::unique_ptr<Plan> g(plan_create(spec, gdims, ho));
+    const int rz = g->an.radius[0];
+    std::unique_ptr<Dist> d(new Dist());
+    d->slab = slab_partition(gdims[0], rz, nranks, rank);
+    d->rz = rz;
+    d->rank = rank;
+    d->nranks = nranks;
+    d->comm = comm;
+    const int64_t ldims[3] = {d->slab.nz_alloc, gdims[1], gdims[2]};
+    d->local = plan_create(spec, ldims, o);
+    d->handle.p = d->local;
+    if (!d->local->host_only) {
+        check_cuda(cudaEventCreateWithFlags(&d->ev_ready, cudaEventDisableTiming), "cudaEventCreate");
+        check_cuda(cudaEventCreateWithFlags(&d->ev_halo, cudaEventDisableTiming), "cudaEventCreate");
+    }
+    return d.release();
+}
+
+namespace {
+
+struct Ranges {
+    bool split = true;  // interior/boundary overlap possible
+    int64_t in_lo = 0, in_hi = 0;
+    int64_t b_lo[2] = {0, 0}, b_hi[2] = {0, 0};  // lower / upper boundary bands
+};
+
+Ranges ranges_of(const Dist *d) {
+    const Slab &s = d->slab;
+    const int64_t rz = d->rz;
+    Ranges r;
+    if (rz == 0 || s.nz_own < 2 * rz) {  // nothing to overlap: one launch after the exchange
+        r.split = false;
+        r.b_lo[0] = s.k_lo;
+        r.b_hi[0] = s.k_hi;
+        return r;
+    }
+    r.in_lo = s.has_lower ? 2 * rz : s.k_lo;
+    r.in_hi = s.has_upper ? s.nz_alloc - 2 * rz : s.k_hi;
+    if (s.has_lower) {
+        r.b_lo[0] = std::max<int64_t>(rz, s.k_lo);
+        r.b_hi[0] = std::min<int64_t>(2 * rz, s.k_hi);
+    }
+    if (s.has_upper) {
+        r.b_lo[1] = std::max<int64_t>(s.nz_alloc - 2 * rz, s.k_lo);
+        r.b_hi[1] = std::min<int64_t>(s.nz_alloc - rz, s.k_hi);
+    }
+    return r;
+}
+
+// z-read inputs that need ghost planes
+std::vector<int> halo_arrays(const Dist *d) {
+    std::vector<int> v;
+    const Plan *p = d->local;
+    for (int f = 0; f < p->n3(); f++) {
+        const Formal &fo = p->st.formal(ArgKind::Array3D, f);
+        if (fo.role == Role::In && p->an.arr_radius[f][0] > 0) v.push_back(f);
+    }
+    return v;
+}
+
+void exchange_nccl(Dist *d, double *const *a3, cudaStream_t comm) {
+    if (d->rz == 0 || d->nranks == 1) return;
+    if (!d->comm) throw Error(SDAG_ERR_INVALID_ARG, "multi-rank dist without an NCCL communicator");
+    const NcclApi &N = nccl();
+    const Plan *p = d->local;
+    const size_t plane = size_t(p->dims[1] * p->dims[2]);
+    const size_t cnt = plane * size_t(d->rz);
+    const Halo h = halo_schedule(d->slab, d->rz);
+    auto c = static_cast<ncclComm_t>(d->comm);
+    nck(N.GroupStart(), "ncclGroupStart");
+    for (int f : halo_arrays(d)) {
+        double *a = a3[f];
+        if (h.lo_send >= 0) {
+            nck(N.Send(a + size_t(h.lo_send) * plane, cnt, ncclFloat64, d->rank - 1, c, comm), "ncclSend");
+            nck(N.Recv(a + size_t(h.lo_recv) * plane, cnt, ncclFloat64, d->rank - 1, c, comm), "ncclRecv");
+        }
+        if (h.up_send >= 0) {
+            nck(N.Send(a + size_t(h.up_send) * plane, cnt, ncclFloat64, d->rank + 1, c, comm), "ncclSend");
+            nck(N.Recv(a + size_t(h.up_recv) * plane, cnt, ncclFloat64, d->rank + 1, c, comm), "ncclRecv");
+        }
+    }
+    nck(N.GroupEnd(), "ncclGroupEnd");
+}
+
+void sweep_split(Dist *d, double *const *a3, const double *const *a1, const double *s, cudaStream_t compute,
+                 cudaStream_t comm, bool do_exchange) {
+    Plan *p = d->local;
+    const KernelDesc &k = p->kernel();
+    const Ranges r = ranges_of(d);
+    const bool xchg = do_exchange && d->rz > 0 && d->nranks > 1;
+    if (xchg) {
+        check_cuda(cudaEventRecord(d->ev_ready, compute), "cudaEventRecord");
+        check_cuda(cudaStreamWaitEvent(comm, d->ev_ready, 0), "cudaStreamWaitEvent");
+        exchange_nccl(d, a3, comm);
+        check_cuda(cudaEventRecord(d->ev_halo, comm), "cudaEventRecord");
+    }
+    if (r.split && r.in_hi > r.in_lo) plan_launch(p, k, const_cast<double *const *>(a3), a1, s, 1, r.in_lo, r.in_hi, compute);
+    if (xchg) check_cuda(cudaStreamWaitEvent(compute, d->ev_halo, 0), "cudaStreamWaitEvent");
+    for (int q = 0; q < 2; q++)
+        if (r.b_hi[q] > r.b_lo[q]) plan_launch(p, k, const_cast<double *const *>(a3), a1, s, 1, r.b_lo[q], r.b_hi[q], compute);
+}
+
+cudaStream_t comm_stream(Dist *d, cudaStream_t comm) {
+    if (comm) return comm;
+    if (!d->own_comm) check_cuda(cudaStreamCreateWithFlags(&d->own_comm, cudaStreamNonBlocking), "cudaStreamCreate");
+    return d->own_comm;
+}
+
+}  // namespace
+
+void dist_apply(Dist *d, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns,
+                cudaStream_t compute, cudaStream_t comm) {
+    if (!d) throw Error(SDAG_ERR_INVALID_ARG, "null dist");
+    Plan *p = d->local;
+    if (p->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
+    if (n3 != p->n3() || n1 != p->n1() || ns != p->ns()) throw Error(SDAG_ERR_INVALID_ARG, "argument counts");
+    for (int f = 0; f < n3; f++)
+        if (!a3[f]) throw Error(SDAG_ERR_INVALID_ARG, "null grid array");
+    if (p->kernel().tma)
+        for (int f = 0; f < n3; f++)
+            if (reinterpret_cast<uintptr_t>(a3[f]) % 16) throw Error(SDAG_ERR_INVALID_ARG, "grid arrays must be 16-B aligned");
+    sweep_split(d, a3, a1, s, compute, comm_stream(d, comm), true);
+}
+
+void dist_apply_iterated(Dist *d, double *b0, double *b1, int T, const double *s, int ns, cudaStream_t compute,
+                         cudaStream_t comm) {
+    if (!d) throw Error(SDAG_ERR_INVALID_ARG, "null dist");
+    Plan *p = d->local;
+    if (p->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
+    if (p->n3() != 2 || p->an.n_in != 1 || p->an.n_out != 1 || p->n1() != 0)
+        throw Error(SDAG_ERR_INVALID_ARG, "iterated dist apply needs a 1-input 1-output plan");
+    if (ns != p->ns() || !b0 || !b1 || b0 == b1) throw Error(SDAG_ERR_INVALID_ARG, "bad arguments");
+    int fin = -1, fout = -1;
+    for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
+    cudaStream_t cs = comm_stream(d, comm);
+    double *bufs[2] = {b0, b1};
+    for (int t = 0; t < T; t++) {
+        double *a3[2];
+        a3[fin] = bufs[t & 1];
+        a3[fout] = bufs[(t + 1) & 1];
+        sweep_split(d, a3, nullptr, s, compute, cs, true);
+    }
+}
+
+void dist_apply_iterated_loopback(Dist **ds, int n, double *const *b0, double *const *b1, int T, const double *s,
+                                  int ns, cudaStream_t stream) {
+    if (!ds || n < 1) throw Error(SDAG_ERR_INVALID_ARG, "bad dist list");
+    for (int r = 0; r < n; r++) {
+        if (!ds[r] || ds[r]->rank != r || ds[r]->nranks != n) throw Error(SDAG_ERR_INVALID_ARG, "dists must be ranks 0..n-1");
+        if (ds[r]->local->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
+    }
+    Plan *p0 = ds[0]->local;
+    if (p0->n3() != 2 || p0->an.n_in != 1 || p0->an.n_out != 1 || p0->n1() != 0 || ns != p0->ns())
+        throw Error(SDAG_ERR_INVALID_ARG, "iterated loopback needs a 1-input 1-output plan");
+    int fin = -1, fout = -1;
+    for (int f = 0; f < 2; f++) (p0->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
+    const int64_t rz = ds[0]->rz;
+    const size_t plane = size_t(p0->dims[1] * p0->dims[2]);
+    for (int t = 0; t < T; t++) {
+        auto in = [&](int r) { return (t & 1) ? b1[r] : b0[r]; };
+        auto out = [&](int r) { return (t & 1) ? b0[r] : b1[r]; };
+        if (rz > 0) {
+            for (int r = 0; r < n; r++) {  // the same schedule the NCCL path sends/receives
+                const Halo h = halo_schedule(ds[r]->slab, int(rz));
+                if (h.lo_recv >= 0) {  // from the lower neighbour's upper send band
+                    const Halo hl = halo_schedule(ds[r - 1]->slab, int(rz));
+                    check_cuda(cudaMemcpyAsync(in(r) + size_t(h.lo_recv) * plane, in(r - 1) + size_t(hl.up_send) * plane,
+                                               size_t(rz) * plane * 8, cudaMemcpyDeviceToDevice, stream),
+                               "loopback halo");
+                }
+                if (h.up_recv >= 0) {  // from the upper neighbour's lower send band
+                    const Halo hu = halo_schedule(ds[r + 1]->slab, int(rz));
+                    check_cuda(cudaMemcpyAsync(in(r) + size_t(h.up_recv) * plane, in(r + 1) + size_t(hu.lo_send) * plane,
+                                               size_t(rz) * plane * 8, cudaMemcpyDeviceToDevice, stream),
+                               "loopback halo");
+                }
+            }
+        }
+        for (int r = 0; r < n; r++) {
+            double *a3[2];
+            a3[fin] = in(r);
+            a3[fout] = out(r);
+            sweep_split(ds[r], a3, nullptr, s, stream, stream, false);
+        }
+    }
+}
+
+}  // namespace sdag

@@ -1,0 +1,48 @@
+// kdesc.cuh -- builds a KernelDesc for one instantiation of the sweep skeleton.
+#pragma once
+
+#include <cstdio>
+
+#include "bodies.cuh"
+#include "kernels.hpp"
+#include "sweep.cuh"
+
+namespace sdag {
+
+template <class B, int TX, int TY, int UX, int UY, int PF, bool TMA>
+KernelDesc make_desc(const char *dag, int prio) {
+    using G = dev::Geo<B, TX, TY, UX, UY, PF>;
+    KernelDesc d;
+    d.dag = dag;
+    char buf[96];
+    std::snprintf(buf, sizeof buf, "%s_%dx%d_u%dx%d_pf%d", TMA ? "tma" : "lsu", TX, TY, UX, UY, PF);
+    d.variant = buf;
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_sweep<B, TX, TY, UX, UY, PF, TMA>);
+    d.threads = G::THREADS;
+    d.smem = G::SMEM;
+    d.tx = TX;
+    d.ty = TY;
+    d.ux = UX;
+    d.uy = UY;
+    d.pf = PF;
+    d.tma = TMA;
+    d.nin = B::NIN;
+    d.nout = B::NOUT;
+    d.nio = B::NIO;
+    d.n1d = B::N1D;
+    d.rz = B::RZ;
+    d.ry = B::RY;
+    d.rx = B::RX;
+    d.rzr = dev::ring_rz<B>();
+    d.prio = prio;
+    return d;
+}
+
+// a TMA variant and its LSU twin (same geometry) for unaligned grids
+#define SDAG_PAIR(v, BODY, DAG, TX, TY, UX, UY, PF, PRIO)                          \
+    do {                                                                           \
+        v.push_back(make_desc<dev::BODY, TX, TY, UX, UY, PF, true>(DAG, PRIO));    \
+        v.push_back(make_desc<dev::BODY, TX, TY, UX, UY, PF, false>(DAG, PRIO + 100)); \
+    } while (0)
+
+}  // namespace sdag

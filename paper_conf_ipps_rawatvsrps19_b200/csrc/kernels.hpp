@@ -1,0 +1,24 @@
+// kernels.hpp -- host-side table of the compiled sm_100a sweep kernels.
+#pragma once
+
+#include <string>
+#include <vector>
+
+namespace sdag {
+
+struct KernelDesc {
+    std::string dag;      // registry DAG this kernel evaluates
+    std::string variant;  // "tma_64x16_u1x4_pf2", ...
+    const void *fn = nullptr;
+    int threads = 0, smem = 0;
+    int tx = 0, ty = 0, ux = 0, uy = 0, pf = 0;
+    bool tma = false;
+    int nin = 0, nout = 0, nio = 0, n1d = 0;
+    int rz = 0, ry = 0, rx = 0, rzr = 0;  // body radius and shared-memory ring z-window
+    int prio = 0;                         // heuristic preference (lower first)
+};
+
+// all kernels, in heuristic preference order per DAG
+const std::vector<KernelDesc> &kernel_table();
+
+}  // namespace sdag

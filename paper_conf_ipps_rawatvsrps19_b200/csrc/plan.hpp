@@ -1,0 +1,87 @@
+// plan.hpp -- an immutable plan (a1-a3 results) plus its small mutable caches.
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <map>
+#include <mutex>
+#include <string>
+#include <tuple>
+#include <vector>
+
+#include "ir.hpp"
+#include "kernels.hpp"
+#include "registry.hpp"
+#include "sdag.h"
+
+namespace sdag {
+
+struct Launch {
+    const KernelDesc *k = nullptr;
+    int nchunk = 1, zchunk = 1;
+    int tiles_x = 1, tiles_y = 1;
+};
+
+struct Plan {
+    Stencil st;
+    Analysis an;
+    const RegEntry *reg = nullptr;
+    std::vector<double> extra_scalars;  // plan-time kernel scalars (shift offsets)
+    int64_t dims[3] = {1, 1, 1};        // nz, ny, nx (one problem)
+    int64_t lo[3] = {0, 0, 0}, hi[3] = {0, 0, 0};
+    int device = -1;
+    bool host_only = false;
+    int sm_count = 148;
+    int batch_hint = 1;
+    int tune = 0;
+    std::string force_variant;
+
+    // ABI mapping (per 3D formal kind_index): staged-input slot / output slot / inout slot
+    std::vector<int> in_slot, out_slot, io_slot;
+    std::vector<const KernelDesc *> cands;  // candidate kernels (TMA first)
+    int chosen = -1;                        // index into cands
+    std::string describe_text;
+
+    // mutable caches
+    std::mutex mu;
+    std::map<std::tuple<const void *, int64_t, int64_t, int64_t, int, int>, CUtensorMap> tmaps;
+    std::vector<void *> ws;  // sdag_apply_host workspace (device buffers)
+    std::vector<size_t> ws_bytes;
+
+    ~Plan();
+    const KernelDesc &kernel() const { return *cands[chosen]; }
+    int n3() const { return st.n_of(ArgKind::Array3D); }
+    int n1() const { return st.n_of(ArgKind::Array1D); }
+    int ns() const { return st.n_of(ArgKind::Scalar); }
+    int64_t points() const { return (hi[0] - lo[0]) * (hi[1] - lo[1]) * (hi[2] - lo[2]); }
+    double bytes_per_point() const;
+};
+
+// planner (runtime.cu)
+Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_plan_opts &o);
+void plan_fill_info(Plan *p, sdag_plan_info *info);
+
+// sweep launch over output planes [klo, khi) of each problem (clipped to the
+// interior); all arrays are per-problem [batch][nz][ny][nx].
+void plan_launch(Plan *p, const KernelDesc &k, double *const *arrays3d, const double *const *arrays1d,
+                 const double *scalars, int batch, int64_t klo, int64_t khi, cudaStream_t stream,
+                 const int64_t *dims_override = nullptr);
+void apply(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns, int batch,
+           cudaStream_t stream);
+void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int ns, cudaStream_t stream);
+void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int n1, const double *s, int ns,
+                cudaStream_t stream, int64_t *h2d, int64_t *d2h);
+void check_cuda(cudaError_t e, const char *what);
+
+// process-wide launch counter
+void count_launch();
+int64_t launch_count();
+double measure_fp64_peak(cudaStream_t stream);
+
+}  // namespace sdag
+
+// the opaque C handle (include/sdag.h) wraps a Plan
+struct sdag_plan_s {
+    sdag::Plan *p;
+};

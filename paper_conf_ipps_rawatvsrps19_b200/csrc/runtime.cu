@@ -1,0 +1,610 @@
+// runtime.cu -- a3 planner and a4-a6 runtime: variant choice, TMA descriptor
+// cache, launch geometry, apply / batched / iterated / host-buffer apply.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstring>
+#include <memory>
+#include <sstream>
+
+#include "plan.hpp"
+#include "sweep.cuh"
+
+namespace sdag {
+
+void add_kernels_jacobi7(std::vector<KernelDesc> &);
+void add_kernels_lap25(std::vector<KernelDesc> &);
+void add_kernels_smooth27(std::vector<KernelDesc> &);
+void add_kernels_hypterm(std::vector<KernelDesc> &);
+void add_kernels_rhs4(std::vector<KernelDesc> &);
+void add_kernels_toys(std::vector<KernelDesc> &);
+
+const std::vector<KernelDesc> &kernel_table() {
+    static std::vector<KernelDesc> v = [] {
+        std::vector<KernelDesc> t;
+        add_kernels_jacobi7(t);
+        add_kernels_lap25(t);
+        add_kernels_smooth27(t);
+        add_kernels_hypterm(t);
+        add_kernels_rhs4(t);
+        add_kernels_toys(t);
+        return t;
+    }();
+    return v;
+}
+
+static std::atomic<int64_t> g_launches{0};
+void count_launch() { g_launches++; }
+int64_t launch_count() { return g_launches.load(); }
+
+void check_cuda(cudaError_t e, const char *what) {
+    if (e != cudaSuccess) {
+        (void)cudaGetLastError();
+        throw Error(SDAG_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+    }
+}
+
+Plan::~Plan() {
+    for (void *b : ws)
+        if (b) cudaFree(b);
+}
+
+// Algorithmic HBM bytes per written point (reading R10):
+// 8 B x (inputs over their footprint box + outputs + 2x inouts over the
+// interior + 1D arrays) / interior points.
+double Plan::bytes_per_point() const {
+    const double pts = double(points());
+    if (pts <= 0) return 0.0;
+    double b = 0.0;
+    for (const auto &f : st.formals) {
+        if (f.kind == ArgKind::Array3D) {
+            if (f.role == Role::In) {
+                double box = 1.0;
+                for (int a = 0; a < 3; a++)
+                    box *= double(std::min<int64_t>(dims[a], (hi[a] - lo[a]) + 2 * an.arr_radius[f.kind_index][a]));
+                b += 8.0 * box;
+            } else if (f.role == Role::Out) {
+                b += 8.0 * pts;
+            } else if (f.role == Role::InOut) {
+                b += 16.0 * pts;
+            }
+        } else if (f.kind == ArgKind::Array1D) {
+            b += 8.0 * double(dims[f.axis]);
+        }
+    }
+    return b / pts;
+}
+
+// ---------------------------------------------------------------------------
+// TMA descriptors
+// ---------------------------------------------------------------------------
+
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        check_cuda(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q),
+                   "cudaGetDriverEntryPoint(cuTensorMapEncodeTiled)");
+        if (!p || q != cudaDriverEntryPointSuccess) throw Error(SDAG_ERR_CUDA, "cuTensorMapEncodeTiled not available");
+        return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    }();
+    return fn;
+}
+
+static CUtensorMap tmap_for(Plan *p, const double *ptr, int64_t nx, int64_t ny, int64_t nzt, int bx, int by) {
+    auto key = std::make_tuple((const void *)ptr, nx, ny, nzt, bx, by);
+    {
+        std::lock_guard<std::mutex> g(p->mu);
+        auto it = p->tmaps.find(key);
+        if (it != p->tmaps.end()) return it->second;
+    }
+    CUtensorMap m;
+    cuuint64_t gdim[3] = {cuuint64_t(nx), cuuint64_t(ny), cuuint64_t(nzt)};
+    cuuint64_t gstride[2] = {cuuint64_t(nx * 8), cuuint64_t(nx * ny * 8)};
+    cuuint32_t box[3] = {cuuint32_t(bx), cuuint32_t(by), 1};
+    cuuint32_t estr[3] = {1, 1, 1};
+    CUresult r = get_encode()(&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double *>(ptr), gdim, gstride, box,
+                              estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) throw Error(SDAG_ERR_CUDA, "cuTensorMapEncodeTiled failed (code " + std::to_string(r) + ")");
+    std::lock_guard<std::mutex> g(p->mu);
+    if (p->tmaps.size() > 256) p->tmaps.clear();
+    p->tmaps[key] = m;
+    return m;
+}
+
+// ---------------------------------------------------------------------------
+// planner
+// ---------------------------------------------------------------------------
+
+static int occupancy_of(const Plan *p, const KernelDesc &k) {
+    if (!p->host_only) {
+        int n = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k.fn, k.threads, k.smem) == cudaSuccess && n > 0)
+            return n;
+        (void)cudaGetLastError();
+    }
+    int bySmem = std::max(1, (228 * 1024) / (k.smem + 1024));
+    int byThreads = std::max(1, 2048 / k.threads);
+    return std::min(bySmem, byThreads);
+}
+
+// z-chunking (concurrent streaming): pick the number of chunks that
+// minimises waves x (chunk + ring refill) for this grid.
+static void geometry(const Plan *p, const KernelDesc &k, int batch, int64_t klo, int64_t khi, const int64_t *lo,
+                     const int64_t *hi, Launch &L) {
+    const int64_t nzi = khi - klo;
+    L.tiles_x = int((hi[2] - lo[2] + k.tx - 1) / k.tx);
+    L.tiles_y = int((hi[1] - lo[1] + k.ty - 1) / k.ty);
+    const int64_t tiles = int64_t(L.tiles_x) * L.tiles_y * batch;
+    const int64_t slots = int64_t(p->sm_count) * occupancy_of(p, k);
+    double best = 1e300;
+    int bestn = 1;
+    const int maxn = int(std::min<int64_t>(nzi, std::max<int64_t>(1, 65535 / std::max(batch, 1))));
+    for (int n = 1; n <= std::min(maxn, 512); n++) {
+        const int64_t zc = (nzi + n - 1) / n;
+        const int64_t units = tiles * ((nzi + zc - 1) / zc);
+        const double waves = double((units + slots - 1) / slots);
+        const double cost = waves * double(zc + 2 * k.rzr + 2);
+        if (cost < best - 1e-9) {
+            best = cost;
+            bestn = n;
+        }
+    }
+    L.zchunk = int((nzi + bestn - 1) / bestn);
+    L.nchunk = int((nzi + L.zchunk - 1) / L.zchunk);
+}
+
+static bool tma_ok(const Plan *p, double *const *a3, int64_t nx) {
+    if (nx % 2 != 0) return false;
+    for (int f = 0; f < p->n3(); f++)
+        if (p->in_slot[f] >= 0 && (reinterpret_cast<uintptr_t>(a3[f]) % 16) != 0) return false;
+    return true;
+}
+
+static const KernelDesc &pick_kernel(Plan *p, double *const *a3, int64_t nx) {
+    const KernelDesc &k = p->kernel();
+    if (!k.tma || tma_ok(p, a3, nx)) return k;
+    for (const KernelDesc *c : p->cands)
+        if (!c->tma && c->tx == k.tx && c->ty == k.ty && c->ux == k.ux && c->uy == k.uy && c->pf == k.pf) return *c;
+    throw Error(SDAG_ERR_INVALID_ARG, "arrays are not 16-byte aligned and no LSU variant exists");
+}
+
+void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *const *a1, const double *s, int batch,
+                 int64_t klo, int64_t khi, cudaStream_t stream, const int64_t *dims_override) {
+    const int64_t *dims = dims_override ? dims_override : p->dims;
+    int64_t lo[3], hi[3];
+    for (int a = 0; a < 3; a++) {
+        const int R = p->an.radius[a];
+        lo[a] = R;
+        hi[a] = dims[a] - R;
+    }
+    klo = std::max(klo, lo[0]);
+    khi = std::min(khi, hi[0]);
+    if (khi <= klo || hi[1] <= lo[1] || hi[2] <= lo[2]) return;  // nothing to compute
+
+    dev::SweepArgs A;
+    std::memset(&A, 0, sizeof A);
+    const int nzt = int(dims[0] * batch);
+    for (int f = 0; f < p->n3(); f++) {
+        const Formal &fo = p->st.formal(ArgKind::Array3D, f);
+        if (p->in_slot[f] >= 0) {
+            A.in[p->in_slot[f]] = a3[f];
+            if (k.tma) A.tmap[p->in_slot[f]] = tmap_for(p, a3[f], dims[2], dims[1], nzt, k.tx + 2 * k.rx, k.ty + 2 * k.ry);
+        }
+        if (p->out_slot[f] >= 0) A.out[p->out_slot[f]] = a3[f];
+        if (p->io_slot[f] >= 0) A.io[p->io_slot[f]] = a3[f];
+        (void)fo;
+    }
+    for (int f = 0; f < p->n1(); f++) {
+        A.a1d[f] = a1[f];
+        A.a1d_bstride[f] = (batch > 1) ? dims[p->st.formal(ArgKind::Array1D, f).axis] : 0;
+    }
+    int ns = 0;
+    for (int q = 0; q < p->ns(); q++) A.s[ns++] = s[q];
+    for (double e : p->extra_scalars) A.s[ns++] = e;
+    A.nx = dims[2];
+    A.ny = dims[1];
+    A.nz = dims[0];
+    A.lo[0] = int32_t(klo);
+    A.hi[0] = int32_t(khi);
+    for (int a = 1; a < 3; a++) {
+        A.lo[a] = int32_t(lo[a]);
+        A.hi[a] = int32_t(hi[a]);
+    }
+    Launch L;
+    int64_t zlo[3] = {klo, lo[1], lo[2]}, zhi[3] = {khi, hi[1], hi[2]};
+    geometry(p, k, batch, klo, khi, zlo, zhi, L);
+    A.tiles_x = L.tiles_x;
+    A.tiles_y = L.tiles_y;
+    A.nchunk = L.nchunk;
+    A.zchunk = L.zchunk;
+
+    static std::mutex attr_mu;
+    static std::map<const void *, int> attr_done;
+    {
+        std::lock_guard<std::mutex> g(attr_mu);
+        int &d = attr_done[k.fn];
+        if (d < k.smem) {
+            check_cuda(cudaFuncSetAttribute(k.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, k.smem),
+                       "cudaFuncSetAttribute(max dynamic smem)");
+            d = k.smem;
+        }
+    }
+    dim3 grid(L.tiles_x, L.tiles_y, L.nchunk * batch);
+    if (grid.z > 65535 || grid.y > 65535) throw Error(SDAG_ERR_DOMAIN, "grid too large (batch x chunks > 65535)");
+    void *args[] = {&A};
+    check_cuda(cudaLaunchKernel(k.fn, grid, dim3(k.threads), args, size_t(k.smem), stream), "sweep launch");
+    count_launch();
+}
+
+static void validate_arrays(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, int ns,
+                            int64_t elems3) {
+    if (n3 != p->n3()) throw Error(SDAG_ERR_INVALID_ARG, "expected " + std::to_string(p->n3()) + " grid arrays");
+    if (n1 != p->n1()) throw Error(SDAG_ERR_INVALID_ARG, "expected " + std::to_string(p->n1()) + " 1D arrays");
+    if (ns != p->ns()) throw Error(SDAG_ERR_INVALID_ARG, "expected " + std::to_string(p->ns()) + " scalars");
+    for (int f = 0; f < n3; f++) {
+        if (!a3 || !a3[f]) throw Error(SDAG_ERR_INVALID_ARG, "null grid array #" + std::to_string(f));
+        if (reinterpret_cast<uintptr_t>(a3[f]) % 8) throw Error(SDAG_ERR_INVALID_ARG, "grid array not 8-byte aligned");
+    }
+    for (int f = 0; f < n1; f++)
+        if (!a1 || !a1[f]) throw Error(SDAG_ERR_INVALID_ARG, "null 1D array #" + std::to_string(f));
+    // outputs may not alias any other array (reading R19)
+    const uintptr_t bytes = uintptr_t(elems3) * 8;
+    for (int f = 0; f < n3; f++) {
+        const Formal &fo = p->st.formal(ArgKind::Array3D, f);
+        if (fo.role != Role::Out && fo.role != Role::InOut) continue;
+        const uintptr_t o0 = reinterpret_cast<uintptr_t>(a3[f]), o1 = o0 + bytes;
+        for (int g = 0; g < n3; g++) {
+            if (g == f) continue;
+            const uintptr_t i0 = reinterpret_cast<uintptr_t>(a3[g]), i1 = i0 + bytes;
+            if (o0 < i1 && i0 < o1)
+                throw Error(SDAG_ERR_INVALID_ARG, "output '" + fo.name + "' overlaps array '" +
+                                                      p->st.formal(ArgKind::Array3D, g).name + "'");
+        }
+    }
+}
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(const Plan *p) {
+        if (p->host_only) throw Error(SDAG_ERR_DEVICE, "plan was created host-only (SDAG_DEVICE_NONE)");
+        check_cuda(cudaGetDevice(&prev), "cudaGetDevice");
+        if (prev != p->device) check_cuda(cudaSetDevice(p->device), "cudaSetDevice");
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+void apply(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns, int batch,
+           cudaStream_t stream) {
+    if (batch < 1) throw Error(SDAG_ERR_INVALID_ARG, "batch must be >= 1");
+    validate_arrays(p, a3, n3, a1, n1, ns, p->dims[0] * p->dims[1] * p->dims[2] * batch);
+    if (ns > 0 && !s) throw Error(SDAG_ERR_INVALID_ARG, "null scalars");
+    DeviceGuard g(p);
+    const KernelDesc &k = pick_kernel(p, a3, p->dims[2]);
+    plan_launch(p, k, a3, a1, s, batch, 0, p->dims[0], stream);
+}
+
+void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int ns, cudaStream_t stream) {
+    if (p->n3() != 2 || p->an.n_in != 1 || p->an.n_out != 1 || p->n1() != 0)
+        throw Error(SDAG_ERR_INVALID_ARG, "apply_iterated needs a 1-input 1-output plan without 1D arrays");
+    if (T < 0) throw Error(SDAG_ERR_INVALID_ARG, "T must be >= 0");
+    if (!b0 || !b1 || b0 == b1) throw Error(SDAG_ERR_INVALID_ARG, "two distinct buffers required");
+    int fin = -1, fout = -1;
+    for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
+    double *bufs[2] = {b0, b1};
+    for (int t = 0; t < T; t++) {
+        double *a3[2];
+        a3[fin] = bufs[t & 1];
+        a3[fout] = bufs[(t + 1) & 1];
+        apply(p, a3, 2, nullptr, 0, s, ns, 1, stream);
+    }
+}
+
+void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int n1, const double *s, int ns,
+                cudaStream_t stream, int64_t *h2d, int64_t *d2h) {
+    const int64_t elems = p->dims[0] * p->dims[1] * p->dims[2];
+    if (n3 != p->n3() || n1 != p->n1() || ns != p->ns()) throw Error(SDAG_ERR_INVALID_ARG, "argument counts");
+    DeviceGuard g(p);
+    {
+        std::lock_guard<std::mutex> lk(p->mu);
+        if (p->ws.empty()) {
+            p->ws.assign(n3 + n1, nullptr);
+            p->ws_bytes.assign(n3 + n1, 0);
+            for (int f = 0; f < n3; f++) {
+                p->ws_bytes[f] = size_t(elems) * 8;
+                check_cuda(cudaMalloc(&p->ws[f], p->ws_bytes[f]), "cudaMalloc(workspace)");
+            }
+            for (int f = 0; f < n1; f++) {
+                p->ws_bytes[n3 + f] = size_t(p->dims[p->st.formal(ArgKind::Array1D, f).axis]) * 8;
+                check_cuda(cudaMalloc(&p->ws[n3 + f], p->ws_bytes[n3 + f]), "cudaMalloc(workspace)");
+            }
+        }
+    }
+    int64_t up = 0, down = 0;
+    std::vector<double *> d3(n3);
+    std::vector<const double *> d1(n1);
+    for (int f = 0; f < n3; f++) {
+        d3[f] = static_cast<double *>(p->ws[f]);
+        const Role r = p->st.formal(ArgKind::Array3D, f).role;
+        if (r == Role::In || r == Role::InOut) {
+            check_cuda(cudaMemcpyAsync(d3[f], h3[f], p->ws_bytes[f], cudaMemcpyHostToDevice, stream), "H2D");
+            up += int64_t(p->ws_bytes[f]);
+        }
+    }
+    for (int f = 0; f < n1; f++) {
+        d1[f] = static_cast<const double *>(p->ws[n3 + f]);
+        check_cuda(cudaMemcpyAsync(p->ws[n3 + f], h1[f], p->ws_bytes[n3 + f], cudaMemcpyHostToDevice, stream), "H2D");
+        up += int64_t(p->ws_bytes[n3 + f]);
+    }
+    apply(p, d3.data(), n3, d1.data(), n1, s, ns, 1, stream);
+    // copy back the written interior box only, so the host ring stays untouched
+    for (int f = 0; f < n3; f++) {
+        const Role r = p->st.formal(ArgKind::Array3D, f).role;
+        if (r != Role::Out && r != Role::InOut) continue;
+        cudaMemcpy3DParms c;
+        std::memset(&c, 0, sizeof c);
+        const size_t nx = size_t(p->dims[2]), ny = size_t(p->dims[1]), nz = size_t(p->dims[0]);
+        c.srcPtr = make_cudaPitchedPtr(d3[f], nx * 8, nx, ny);
+        c.dstPtr = make_cudaPitchedPtr(h3[f], nx * 8, nx, ny);
+        c.srcPos = make_cudaPos(size_t(p->lo[2]) * 8, size_t(p->lo[1]), size_t(p->lo[0]));
+        c.dstPos = c.srcPos;
+        c.extent = make_cudaExtent(size_t(p->hi[2] - p->lo[2]) * 8, size_t(p->hi[1] - p->lo[1]),
+                                   size_t(p->hi[0] - p->lo[0]));
+        c.kind = cudaMemcpyDeviceToHost;
+        (void)nz;
+        check_cuda(cudaMemcpy3DAsync(&c, stream), "D2H");
+        down += int64_t(c.extent.width) * int64_t(c.extent.height) * int64_t(c.extent.depth);
+    }
+    check_cuda(cudaStreamSynchronize(stream), "cudaStreamSynchronize");
+    if (h2d) *h2d = up;
+    if (d2h) *d2h = down;
+}
+
+// ---------------------------------------------------------------------------
+// plan creation
+// ---------------------------------------------------------------------------
+
+static void time_candidates(Plan *p);
+
+Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_plan_opts &o) {
+    std::unique_ptr<Plan> p(new Plan());
+    p->st = parse_spec(spec);                 // a1
+    p->an = analyse(p->st);                   // a2
+    const int nit = int(p->st.iterators.size());
+    for (int a = 0; a < 3; a++) {
+        if (dims[a] < 1) throw Error(SDAG_ERR_DOMAIN, "dims must be >= 1");
+        if (a < 3 - nit && dims[a] != 1)
+            throw Error(SDAG_ERR_DOMAIN, "a " + std::to_string(nit) + "-iterator spec needs leading dims of 1");
+        if (dims[a] > (int64_t(1) << 30)) throw Error(SDAG_ERR_DOMAIN, "extent too large");
+        p->dims[a] = dims[a];
+        const int R = p->an.radius[a];
+        if (o.order >= 0 && R > o.order)
+            throw Error(SDAG_ERR_DOMAIN, "an access reaches radius " + std::to_string(R) + " > declared order " +
+                                             std::to_string(o.order));
+        if (dims[a] < 2 * R + 1)
+            throw Error(SDAG_ERR_DOMAIN, "extent " + std::to_string(dims[a]) + " has no interior for radius " +
+                                             std::to_string(R));
+        p->lo[a] = R;
+        p->hi[a] = dims[a] - R;
+    }
+    // a3: bind to a registered sm_100a body
+    p->reg = match_dag(p->st, p->extra_scalars);
+    // ABI slots: staged inputs, outputs and inouts in formal order
+    const int n3 = p->n3();
+    p->in_slot.assign(n3, -1);
+    p->out_slot.assign(n3, -1);
+    p->io_slot.assign(n3, -1);
+    int ni = 0, no = 0, nio = 0;
+    for (int f = 0; f < n3; f++) {
+        const Role r = p->st.formal(ArgKind::Array3D, f).role;
+        if (r == Role::In) p->in_slot[f] = ni++;
+        if (r == Role::Out || r == Role::InOut) p->out_slot[f] = no++;
+        if (r == Role::InOut) p->io_slot[f] = nio++;
+    }
+    p->batch_hint = std::max(1, o.batch);
+    p->tune = o.tune;
+    if (o.force_variant) p->force_variant = o.force_variant;
+
+    // device
+    if (o.device == SDAG_DEVICE_NONE) {
+        p->host_only = true;
+        p->sm_count = 148;
+    } else {
+        int ndev = 0;
+        cudaError_t e = cudaGetDeviceCount(&ndev);
+        if (e != cudaSuccess || ndev == 0) {
+            (void)cudaGetLastError();
+            throw Error(SDAG_ERR_DEVICE, "no CUDA device (sdag has no CPU fallback)");
+        }
+        int dev = o.device;
+        if (dev < 0) check_cuda(cudaGetDevice(&dev), "cudaGetDevice");
+        if (dev >= ndev) throw Error(SDAG_ERR_DEVICE, "device ordinal out of range");
+        cudaDeviceProp prop;
+        check_cuda(cudaGetDeviceProperties(&prop, dev), "cudaGetDeviceProperties");
+        if (prop.major != 10 || prop.minor != 0)
+            throw Error(SDAG_ERR_DEVICE, std::string("sdag kernels are built for sm_100a; device is ") + prop.name +
+                                             " sm_" + std::to_string(prop.major) + std::to_string(prop.minor));
+        p->device = dev;
+        p->sm_count = prop.multiProcessorCount;
+    }
+
+    std::ostringstream d;
+    d << "stencil '" << p->st.name << "' -> dag '" << (p->reg ? p->reg->name : std::string("(unregistered)"))
+      << "'\n"
+      << "  radius (z,y,x) = (" << p->an.radius[0] << "," << p->an.radius[1] << "," << p->an.radius[2] << ")"
+      << "  flops/pt = " << p->an.flops_per_point << "  bytes/pt = " << p->bytes_per_point()
+      << "  IO arrays = " << p->an.n_io_arrays << "  homogenizable(z) = " << (p->an.homogenizable_z ? "yes" : "no");
+    if (!p->reg) {
+        // analysis-only plans are allowed host-only; a device plan needs a kernel
+        if (!p->host_only)
+            throw Error(SDAG_ERR_UNSUPPORTED, "no sm_100a kernel is registered for this stencil DAG (registered: " +
+                                                  registry_names() + "); arbitrary DAG code generation is NEXT-4");
+        d << "\n  no registered sm_100a body (analysis only)";
+        p->describe_text = d.str();
+        return p.release();
+    }
+
+    // candidates: kernels of this DAG, TMA variants only when nx is even
+    for (const KernelDesc &k : kernel_table()) {
+        if (k.dag != p->reg->name) continue;
+        if (k.tma && p->dims[2] % 2 != 0) continue;
+        if (k.smem > 227 * 1024) continue;
+        p->cands.push_back(&k);
+    }
+    std::stable_sort(p->cands.begin(), p->cands.end(),
+                     [](const KernelDesc *a, const KernelDesc *b) { return a->prio < b->prio; });
+    if (p->cands.empty()) throw Error(SDAG_ERR_UNSUPPORTED, "no kernel variant fits this plan");
+    p->chosen = 0;
+    if (!p->force_variant.empty()) {
+        p->chosen = -1;
+        for (size_t q = 0; q < p->cands.size(); q++)
+            if (p->cands[q]->variant == p->force_variant) p->chosen = int(q);
+        if (p->chosen < 0) throw Error(SDAG_ERR_INVALID_ARG, "unknown variant '" + p->force_variant + "'");
+    } else if (p->tune && !p->host_only) {
+        time_candidates(p.get());
+    }
+
+    const KernelDesc &k = p->kernel();
+    d << "\n  variant " << k.variant << " (" << k.threads << " threads, " << k.smem << " B smem, ring "
+      << (2 * k.rzr + 1 + k.pf) << " planes)" << (p->tune ? "  [tuned]" : "  [heuristic]") << "\n  candidates:";
+    for (auto *c : p->cands) d << " " << c->variant;
+    p->describe_text = d.str();
+    return p.release();
+}
+
+// Hierarchical autotuning, lite: time every candidate geometry on
+// scratch buffers of the plan's shape and keep the fastest.
+static void time_candidates(Plan *p) {
+    DeviceGuard g(p);
+    const int64_t elems = p->dims[0] * p->dims[1] * p->dims[2] * p->batch_hint;
+    std::vector<double *> b3(p->n3(), nullptr);
+    std::vector<const double *> b1(p->n1(), nullptr);
+    std::vector<void *> owned;
+    auto cleanup = [&] {
+        for (void *q : owned) cudaFree(q);
+    };
+    try {
+        for (int f = 0; f < p->n3(); f++) {
+            void *q;
+            check_cuda(cudaMalloc(&q, size_t(elems) * 8), "cudaMalloc(tune)");
+            check_cuda(cudaMemset(q, 0, size_t(elems) * 8), "cudaMemset(tune)");
+            owned.push_back(q);
+            b3[f] = static_cast<double *>(q);
+        }
+        for (int f = 0; f < p->n1(); f++) {
+            void *q;
+            const size_t n = size_t(p->dims[p->st.formal(ArgKind::Array1D, f).axis]) * p->batch_hint * 8;
+            check_cuda(cudaMalloc(&q, n), "cudaMalloc(tune)");
+            check_cuda(cudaMemset(q, 0, n), "cudaMemset(tune)");
+            owned.push_back(q);
+            b1[f] = static_cast<const double *>(q);
+        }
+        std::vector<double> s(std::max(1, p->ns()), 1.0);
+        cudaEvent_t e0, e1;
+        check_cuda(cudaEventCreate(&e0), "event");
+        check_cuda(cudaEventCreate(&e1), "event");
+        float best = 1e30f;
+        int bestq = 0;
+        for (size_t q = 0; q < p->cands.size() && q < 16; q++) {
+            const KernelDesc &k = *p->cands[q];
+            if (!k.tma && p->dims[2] % 2 == 0) continue;  // LSU twins only matter for odd nx
+            plan_launch(p, k, b3.data(), b1.data(), s.data(), p->batch_hint, 0, p->dims[0], 0);
+            check_cuda(cudaEventRecord(e0, 0), "event");
+            for (int r = 0; r < 3; r++)
+                plan_launch(p, k, b3.data(), b1.data(), s.data(), p->batch_hint, 0, p->dims[0], 0);
+            check_cuda(cudaEventRecord(e1, 0), "event");
+            check_cuda(cudaEventSynchronize(e1), "event sync");
+            float ms = 0;
+            check_cuda(cudaEventElapsedTime(&ms, e0, e1), "event time");
+            if (ms < best) {
+                best = ms;
+                bestq = int(q);
+            }
+        }
+        cudaEventDestroy(e0);
+        cudaEventDestroy(e1);
+        p->chosen = bestq;
+    } catch (...) {
+        cleanup();
+        throw;
+    }
+    cleanup();
+}
+
+void plan_fill_info(Plan *p, sdag_plan_info *info) {
+    std::memset(info, 0, sizeof *info);
+    info->n_arrays3d = p->n3();
+    info->n_arrays1d = p->n1();
+    info->n_scalars = p->ns();
+    info->n_in = p->an.n_in;
+    info->n_out = p->an.n_out;
+    info->n_inout = p->an.n_inout;
+    info->n_statements = int(p->st.stmts.size());
+    info->n_temporaries = int(p->st.temps.size());
+    for (int a = 0; a < 3; a++) {
+        info->radius[a] = p->an.radius[a];
+        info->dims[a] = p->dims[a];
+        info->lo[a] = p->lo[a];
+        info->hi[a] = p->hi[a];
+    }
+    info->points = p->points();
+    info->flops_per_point = p->an.flops_per_point;
+    info->bytes_per_point = p->bytes_per_point();
+    info->oi_paper = p->an.n_io_arrays ? p->an.flops_per_point / (8.0 * p->an.n_io_arrays) : 0.0;
+    info->n_kernels = 1;
+    info->n_variants = int(p->cands.size());
+    info->dag = p->reg ? p->reg->name.c_str() : "";
+    info->variant = p->cands.empty() ? "" : p->kernel().variant.c_str();
+    if (p->cands.empty()) info->n_kernels = 0;
+}
+
+// ---------------------------------------------------------------------------
+// FP64 peak micro-benchmark: independent DFMA chains on every SM
+// ---------------------------------------------------------------------------
+
+__global__ void __launch_bounds__(256) sdag_fp64_peak(double *out, int iters, double a, double b) {
+    double x[8];
+#pragma unroll
+    for (int q = 0; q < 8; q++) x[q] = threadIdx.x * 1e-3 + q;
+    for (int it = 0; it < iters; it++) {
+#pragma unroll
+        for (int q = 0; q < 8; q++) x[q] = fma(x[q], a, b);
+    }
+    double s = 0;
+#pragma unroll
+    for (int q = 0; q < 8; q++) s += x[q];
+    if (s == 12345.678) out[0] = s;  // never true; keeps the chains alive
+}
+
+double measure_fp64_peak(cudaStream_t stream) {
+    int dev = 0, sms = 0;
+    check_cuda(cudaGetDevice(&dev), "cudaGetDevice");
+    check_cuda(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev), "attr");
+    double *out = nullptr;
+    check_cuda(cudaMalloc(&out, 8), "cudaMalloc");
+    const int blocks = sms * 8, iters = 1 << 14;
+    cudaEvent_t e0, e1;
+    check_cuda(cudaEventCreate(&e0), "event");
+    check_cuda(cudaEventCreate(&e1), "event");
+    sdag_fp64_peak<<<blocks, 256, 0, stream>>>(out, 256, 0.999999, 1e-7);
+    check_cuda(cudaEventRecord(e0, stream), "event");
+    sdag_fp64_peak<<<blocks, 256, 0, stream>>>(out, iters, 0.999999, 1e-7);
+    check_cuda(cudaEventRecord(e1, stream), "event");
+    check_cuda(cudaEventSynchronize(e1), "sync");
+    float ms = 0;
+    check_cuda(cudaEventElapsedTime(&ms, e0, e1), "elapsed");
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(out);
+    const double flops = 2.0 * 8.0 * double(iters) * double(blocks) * 256.0;
+    return flops / (double(ms) * 1e-3);
+}
+
+}  // namespace sdag

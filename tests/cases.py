@@ -1,0 +1,108 @@
+"""Shared helpers for the GPU parity tests: run a registered DAG through the
+C ABI (paper_conf_ipps_rawatvsrps19_b200) and through the CPU oracle on the
+same seeded inputs, and compare with the scaled-error gate of DESIGN.md
+reading R13:  e_p = |g_p - o_p| / max(|o_p|, A_p) <= TOL, A_p the abs-mode
+oracle value."""
+from __future__ import annotations
+
+import numpy as np
+
+import oracle
+import synth
+
+TOL = 1e-12  # BASELINE.json north_star: "max relative error 1e-12" (reading R13)
+
+RADIUS = {"jacobi7": 1, "lap25": 4, "smooth27": 1, "hypterm": 4, "rhs4center": 2}
+
+
+def interior(shape, R):
+    return tuple(slice(R, n - R) for n in shape)
+
+
+def ring_mask(shape, R):
+    m = np.ones(shape, dtype=bool)
+    m[interior(shape, R)] = False
+    return m
+
+
+def scaled_err(g, o, a):
+    g, o, a = np.asarray(g), np.asarray(o), np.asarray(a)
+    den = np.maximum(np.abs(o), a)
+    with np.errstate(invalid="ignore", divide="ignore"):
+        e = np.where(den > 0, np.abs(g - o) / np.where(den > 0, den, 1.0), np.abs(g - o))
+    return float(np.max(e)) if e.size else 0.0
+
+
+def make_case(name, dims, cfg="t"):
+    """-> dict(inputs (formal-order lists), scalars, oracle outputs, abs-mode outputs)"""
+    if name == "jacobi7":
+        ins, sc = synth.jacobi7_inputs(dims, cfg=cfg)
+        A = ins["A"]
+        s_abi = [sc["h2inv"], sc["a"], sc["b"]]
+        o = [oracle.jacobi7(A, sc["a"], sc["b"], sc["h2inv"])]
+        a = [oracle.jacobi7(np.abs(A), abs(sc["a"]), abs(sc["b"]), abs(sc["h2inv"]), absmode=True)]
+        return dict(inputs=[A], outs=1, s=s_abi, a1d=[], o=o, a=a, inout=[])
+    if name == "lap25":
+        ins, sc = synth.lap25_inputs(dims, cfg=cfg)
+        A = ins["A"]
+        c = [sc[k] for k in ("c0", "c1", "c2", "c3", "c4")]
+        return dict(inputs=[A], outs=1, s=c, a1d=[], o=[oracle.lap25(A, c)],
+                    a=[oracle.lap25(np.abs(A), np.abs(c), absmode=True)], inout=[])
+    if name == "smooth27":
+        ins, sc = synth.smooth27_inputs(dims, cfg=cfg)
+        A = ins["A"]
+        w = [sc[k] for k in ("w0", "w1", "w2", "w3")]
+        return dict(inputs=[A], outs=1, s=[*w, sc["nu"]], a1d=[], o=[oracle.smooth27(A, w, sc["nu"])],
+                    a=[oracle.smooth27(np.abs(A), np.abs(w), abs(sc["nu"]), absmode=True)], inout=[])
+    if name == "hypterm":
+        ins, sc = synth.hypterm_inputs(dims, cfg=cfg)
+        arrs = [ins[k] for k in ("cons_1", "cons_2", "cons_3", "cons_4", "q_1", "q_2", "q_3", "q_4")]
+        s = [sc[k] for k in ("dxinv0", "dxinv1", "dxinv2", "ALP", "BET", "GAM", "DEL")]
+        o = oracle.hypterm(arrs, s[:3], s[3:])
+        a = oracle.hypterm([np.abs(x) for x in arrs], np.abs(s[:3]), np.abs(s[3:]), absmode=True)
+        return dict(inputs=arrs, outs=5, s=s, a1d=[], o=o, a=a, inout=[])
+    if name == "rhs4center":
+        ins, sc = synth.rhs4_inputs(dims, cfg=cfg)
+        u = [ins["u0"], ins["u1"], ins["u2"]]
+        ua = [ins["uacc0"], ins["uacc1"], ins["uacc2"]]
+        s = [sc[k] for k in ("tf", "i6", "i144", "cof", "a1")]
+        a1d = [ins["strx"], ins["stry"], ins["strz"]]
+        o = oracle.rhs4(u, ins["mu"], ins["la"], *a1d, ua, *s)
+        a = oracle.rhs4([np.abs(x) for x in u], np.abs(ins["mu"]), np.abs(ins["la"]), *[np.abs(x) for x in a1d],
+                        [np.abs(x) for x in ua], *np.abs(s), absmode=True)
+        return dict(inputs=[*u, ins["mu"], ins["la"]], outs=0, s=s, a1d=a1d, o=o, a=a, inout=ua)
+    raise KeyError(name)
+
+
+def run_gpu(name, dims, case, variant=None, tune=False, sentinel=np.nan):
+    """Apply through the C ABI; 3D formals in the registered spec's order.
+    Returns the written arrays (outputs, or inouts) as numpy."""
+    import torch
+
+    import paper_conf_ipps_rawatvsrps19_b200 as sdag
+    plan = sdag.Plan(sdag.spec_text(name), dims, variant=variant, tune=tune)
+    dev = [torch.from_numpy(np.ascontiguousarray(x)).cuda() for x in case["inputs"]]
+    if case["inout"]:
+        outs = [torch.from_numpy(x.copy()).cuda() for x in case["inout"]]
+    else:
+        outs = [torch.full(tuple(dims), sentinel, dtype=torch.float64, device="cuda") for _ in range(case["outs"])]
+    a1d = [torch.from_numpy(x).cuda() for x in case["a1d"]]
+    plan.apply(outs + dev, a1d, case["s"])
+    torch.cuda.synchronize()
+    return [t.cpu().numpy() for t in outs], plan
+
+
+def check(name, dims, g, case):
+    R = RADIUS[name]
+    I = interior(dims, R)
+    worst = 0.0
+    for m, (gm, om, am) in enumerate(zip(g, case["o"], case["a"])):
+        e = scaled_err(gm[I], om[I], am[I])
+        worst = max(worst, e)
+        assert e <= TOL, f"{name} output {m}: scaled error {e:.3e} > {TOL}"
+        ring = ring_mask(dims, R)
+        if case["inout"]:
+            assert np.array_equal(gm[ring], case["inout"][m][ring]), f"{name} output {m}: ring modified"
+        else:
+            assert np.all(np.isnan(gm[ring])), f"{name} output {m}: wrote outside the interior"
+    return worst
