@@ -5,6 +5,7 @@
 
 #include "bodies.cuh"
 #include "kernels.hpp"
+#include "star.cuh"
 #include "sweep.cuh"
 
 namespace sdag {
@@ -37,6 +38,40 @@ KernelDesc make_desc(const char *dag, int prio) {
     d.prio = prio;
     return d;
 }
+
+// star-stencil kernel (star.cuh): 2-wide x patch, UY-tall y patch, register z-queue
+template <class B, int TX, int TY, int UY, int PF, bool TMA>
+KernelDesc make_star_desc(const char *dag, int prio) {
+    using G = dev::StarGeo<B, TX, TY, UY, PF>;
+    KernelDesc d;
+    d.dag = dag;
+    char buf[96];
+    std::snprintf(buf, sizeof buf, "star_%s_%dx%d_u2x%d_pf%d", TMA ? "tma" : "lsu", TX, TY, UY, PF);
+    d.variant = buf;
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_star<B, TX, TY, UY, PF, TMA>);
+    d.threads = G::THREADS;
+    d.smem = G::SMEM;
+    d.tx = TX;
+    d.ty = TY;
+    d.ux = 2;
+    d.uy = UY;
+    d.pf = PF;
+    d.tma = TMA;
+    d.nin = 1;
+    d.nout = 1;
+    d.rz = B::R;
+    d.ry = B::R;
+    d.rx = G::ML;  // TMA box margin in x (R rounded up to even)
+    d.rzr = B::R;
+    d.prio = prio;
+    return d;
+}
+
+#define SDAG_STAR_PAIR(v, BODY, DAG, TX, TY, UY, PF, PRIO)                                \
+    do {                                                                                   \
+        v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true>(DAG, PRIO));           \
+        v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, false>(DAG, PRIO + 100));    \
+    } while (0)
 
 // a TMA variant and its LSU twin (same geometry) for unaligned grids
 #define SDAG_PAIR(v, BODY, DAG, TX, TY, UX, UY, PF, PRIO)                          \

@@ -1,0 +1,236 @@
+// star.cuh -- sm_100a z-streaming kernel for axis-aligned star stencils
+// (Listing 1's 7-point Jacobi, the 25-point radius-4 Laplacian).
+//
+// B200 design: the HBM roofline leaves ~0.7 SM
+// clocks per output point, i.e. <= ~90 B of shared-memory traffic per point at
+// 128 B/clk/SM, so the generic skeleton's all-taps-from-smem evaluation
+// (~19 doubles/point for R=4) is shared-memory bound.  This kernel keeps
+//  * the z-taps in a per-thread register queue of 2R+1 plane values
+//    (serial streaming with register reuse along the streamed dimension,
+//    P:611-638; the retiming idea of P:790-830 applied to the centre column),
+//  * a 2-wide x patch read with 128-bit LDS (blocked unrolling):
+//    each row window [x-R, x+2+R) is (R+1) aligned double2 loads,
+//  * a UY-tall y patch whose column [y-R, y+UY+R) is read once per plane,
+// so each point costs ~9 doubles of smem reads for R=4 (4.5 for R=1).
+// Planes arrive by TMA (cp.async.bulk.tensor.3d + mbarrier expect_tx) into a
+// ring of R+1+PF slots: plane p is used first as the queue head (its centre
+// values) and last, R iterations later, as the centre plane with its xy halo.
+//
+// Arithmetic is re-associated relative to the spec (y/z taps first, then x,
+// then the centre, each group as fma(c_r, sum, acc)); parity is by the scaled
+// error gate (reading R13).
+#pragma once
+
+#include "sweep.cuh"
+
+namespace sdag {
+namespace dev {
+
+// 25-point radius-4 Laplacian: B = c0*A + sum_r c_r*(6 taps at distance r)
+struct Lap25Star {
+    static constexpr int R = 4, NIN = 1, NOUT = 1, NIO = 0, N1D = 0, RZ = 4, RY = 4, RX = 4, RZR = 4;
+    __host__ __device__ static constexpr int axis1d(int) { return 2; }
+    __device__ __forceinline__ static void yz(double &acc, const SweepArgs &a, int r, double s) {
+        acc = fma(a.s[r], s, acc);
+    }
+    __device__ __forceinline__ static void x(double &acc, const SweepArgs &a, int r, double s) {
+        acc = fma(a.s[r], s, acc);
+    }
+    __device__ __forceinline__ static double finish(double acc, const SweepArgs &a, double ctr) {
+        return fma(a.s[0], ctr, acc);
+    }
+};
+
+// Listing 1: B = a*A - (b*h2inv)*(6 neighbours - 6*A); scalars (h2inv, a, b)
+struct Jacobi7Star {
+    static constexpr int R = 1, NIN = 1, NOUT = 1, NIO = 0, N1D = 0, RZ = 1, RY = 1, RX = 1, RZR = 1;
+    __host__ __device__ static constexpr int axis1d(int) { return 2; }
+    __device__ __forceinline__ static void yz(double &acc, const SweepArgs &, int, double s) { acc += s; }
+    __device__ __forceinline__ static void x(double &acc, const SweepArgs &, int, double s) { acc += s; }
+    __device__ __forceinline__ static double finish(double acc, const SweepArgs &a, double ctr) {
+        const double c = a.s[2] * a.s[0];
+        return a.s[1] * ctr - c * fma(-6.0, ctr, acc);
+    }
+};
+
+template <class B, int TX, int TY, int UY, int PF>
+struct StarGeo {
+    static constexpr int R = B::R;
+    static constexpr int NTX = TX / 2, NTY = TY / UY, THREADS = NTX * NTY;
+    // left/right box margin ML = R rounded up to even, so the centre column
+    // cx + ML and the aligned x-window start cx are both 16-B aligned in smem
+    static constexpr int ML = R + (R % 2);
+    static constexpr int PX = TX + 2 * ML, PY = TY + 2 * R, PLANE = PX * PY;
+    static constexpr int WN = 2 * (R + 1 + (R % 2));  // x-window elements loaded per row (double2 aligned)
+    static constexpr int PLANE_AL = ((PLANE * 8 + 127) / 128) * 128 / 8;
+    static constexpr int NS = R + 1 + PF;  // ring slots
+    static constexpr int NQ = 2 * R + 1;   // register queue depth
+    static constexpr int SMEM = NS * PLANE_AL * 8 + NS * 8;
+    static_assert(TX % 2 == 0 && TY % UY == 0, "tile");
+    static_assert(PX <= 256 && PY <= 256, "TMA box");
+};
+
+template <class B, int TX, int TY, int UY, int PF, bool USE_TMA>
+__global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
+    sdag_star(const __grid_constant__ SweepArgs a) {
+    using G = StarGeo<B, TX, TY, UY, PF>;
+    constexpr int R = G::R, PX = G::PX, NS = G::NS, NQ = G::NQ, PAL = G::PLANE_AL, ML = G::ML, WN = G::WN;
+
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    double *ring = reinterpret_cast<double *>(smem_raw);
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem_raw + NS * PAL * 8);
+
+    const int tile_x = blockIdx.x, tile_y = blockIdx.y;
+    const int chunk = blockIdx.z % a.nchunk;
+    const int64_t prob = blockIdx.z / a.nchunk;
+    const int x0 = a.lo[2] + tile_x * TX, y0 = a.lo[1] + tile_y * TY;
+    const int kb = a.lo[0] + chunk * a.zchunk;
+    const int ke = min(a.hi[0], kb + a.zchunk);
+    if (kb >= ke) return;
+    const int p0 = kb - R, plast = ke - 1 + R;
+    const int64_t zbase = prob * a.nz;
+
+    const int t = threadIdx.x;
+    const int lx = t % G::NTX, ly = t / G::NTX;
+    const int cx = 2 * lx;       // patch x offset inside the tile (even: 16-B aligned in smem)
+    const int cy = UY * ly;      // patch y offset inside the tile
+
+    auto issue = [&](int p) {
+        const int slot = (p - p0) % NS;
+        double *dst = ring + slot * PAL;
+        if constexpr (USE_TMA) {
+            if (t == 0) {
+                mbar_expect_tx(&bars[slot], uint32_t(G::PLANE * 8));
+                tma_load_3d(dst, &a.tmap[0], &bars[slot], x0 - ML, y0 - R, int(zbase + p));
+            }
+        } else {
+            const int64_t pl = (zbase + p) * a.ny * a.nx;
+            for (int e = t; e < G::PLANE; e += G::THREADS) {
+                const int yy = e / PX, xx = e % PX;
+                const int gx = x0 - ML + xx, gy = y0 - R + yy;
+                const bool ok = gx >= 0 && gx < a.nx && gy >= 0 && gy < a.ny && p >= 0 && p < a.nz;
+                cp_async8(dst + e, a.in[0] + (ok ? pl + int64_t(gy) * a.nx + gx : 0), ok);
+            }
+        }
+    };
+    auto wait = [&](int p) {
+        if constexpr (USE_TMA) {
+            mbar_wait(&bars[(p - p0) % NS], ((p - p0) / NS) & 1);
+        } else {
+            cp_async_wait<PF>();
+            __syncthreads();
+        }
+    };
+
+    if constexpr (USE_TMA) {
+        if (t == 0) {
+            for (int s = 0; s < NS; s++) mbar_init(&bars[s], 1);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+        __syncthreads();
+    }
+    for (int p = p0; p < p0 + PF; p++) {
+        if (p <= plast) issue(p);
+        if constexpr (!USE_TMA) cp_async_commit();
+    }
+
+    double q[NQ][UY][2];  // q[d] = centre values of plane p-2R+d (d = 2R: newest)
+#pragma unroll
+    for (int d = 0; d < NQ; d++)
+#pragma unroll
+        for (int py = 0; py < UY; py++) q[d][py][0] = q[d][py][1] = 0.0;
+
+    const bool col_in = (x0 + cx) < a.hi[2];
+    for (int p = p0; p <= plast; p++) {
+        {
+            const int pn = p + PF;
+            if (pn <= plast) issue(pn);
+            if constexpr (!USE_TMA) cp_async_commit();
+        }
+        wait(p);
+        // shift the queue and load the head (plane p's centre values)
+#pragma unroll
+        for (int d = 0; d < NQ - 1; d++)
+#pragma unroll
+            for (int py = 0; py < UY; py++) {
+                q[d][py][0] = q[d + 1][py][0];
+                q[d][py][1] = q[d + 1][py][1];
+            }
+        {
+            const double *hp = ring + ((p - p0) % NS) * PAL + (cy + R) * PX + (cx + ML);
+#pragma unroll
+            for (int py = 0; py < UY; py++) {
+                const double2 v = *reinterpret_cast<const double2 *>(hp + py * PX);
+                q[NQ - 1][py][0] = v.x;
+                q[NQ - 1][py][1] = v.y;
+            }
+        }
+        const int k = p - R;
+        if (k >= kb) {
+            const double *cp = ring + ((k - p0) % NS) * PAL;  // centre plane k with its xy halo
+            double acc[UY][2];
+#pragma unroll
+            for (int py = 0; py < UY; py++) acc[py][0] = acc[py][1] = 0.0;
+            // y and z taps: column rows [cy-R, cy+UY+R) of plane k
+            {
+                double col[UY + 2 * R][2];
+#pragma unroll
+                for (int r = 0; r < UY + 2 * R; r++) {
+                    const double2 v = *reinterpret_cast<const double2 *>(cp + (cy + r) * PX + (cx + ML));
+                    col[r][0] = v.x;
+                    col[r][1] = v.y;
+                }
+#pragma unroll
+                for (int py = 0; py < UY; py++)
+#pragma unroll
+                    for (int px = 0; px < 2; px++)
+#pragma unroll
+                        for (int r = 1; r <= R; r++)
+                            B::yz(acc[py][px], a, r,
+                                  (col[py + R + r][px] + col[py + R - r][px]) + (q[R + r][py][px] + q[R - r][py][px]));
+            }
+            // x taps: the row window [cx-R, cx+2+R) lies in the aligned span
+            // [cx, cx+WN) of smem columns; w[ML + px + dx] is the tap (px, dx)
+#pragma unroll
+            for (int py = 0; py < UY; py++) {
+                double w[WN];
+                const double *rp = cp + (cy + py + R) * PX + cx;
+#pragma unroll
+                for (int c = 0; c < WN / 2; c++) {
+                    const double2 v = *reinterpret_cast<const double2 *>(rp + 2 * c);
+                    w[2 * c] = v.x;
+                    w[2 * c + 1] = v.y;
+                }
+#pragma unroll
+                for (int px = 0; px < 2; px++) {
+#pragma unroll
+                    for (int r = 1; r <= R; r++) B::x(acc[py][px], a, r, w[ML + px + r] + w[ML + px - r]);
+                    acc[py][px] = B::finish(acc[py][px], a, w[ML + px]);
+                }
+            }
+            // interior-only streaming stores (2-wide when both points are inside)
+            const int gi = x0 + cx;
+#pragma unroll
+            for (int py = 0; py < UY; py++) {
+                const int gj = y0 + cy + py;
+                if (gj < a.hi[1] && col_in) {
+                    double *o = a.out[0] + ((zbase + k) * a.ny + gj) * a.nx + gi;
+                    if (gi + 1 < a.hi[2]) {
+                        if ((reinterpret_cast<uintptr_t>(o) & 15) == 0)
+                            __stcs(reinterpret_cast<double2 *>(o), make_double2(acc[py][0], acc[py][1]));
+                        else {
+                            __stcs(o, acc[py][0]);
+                            __stcs(o + 1, acc[py][1]);
+                        }
+                    } else {
+                        __stcs(o, acc[py][0]);
+                    }
+                }
+            }
+        }
+        __syncthreads();  // slot of plane k is reused by the next issue
+    }
+}
+
+}  // namespace dev
+}  // namespace sdag
