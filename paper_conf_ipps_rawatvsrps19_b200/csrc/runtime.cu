@@ -216,8 +216,14 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *
         A.lo[a] = int32_t(lo[a]);
         A.hi[a] = int32_t(hi[a]);
     }
+    // The TMA box of a tile starts at (tile x origin - k.rx).  B200's FP64 tiled
+    // TMA traps ("illegal instruction") on a box whose x origin is not 16-byte
+    // aligned (tools/tma_probe.cu), so the tile grid may start one (ring)
+    // column left of the interior; kernels mask x < xmin.
+    A.xmin = int32_t(lo[2]);
+    A.lo[2] = int32_t(lo[2] - ((lo[2] - k.rx) & 1));
     Launch L;
-    int64_t zlo[3] = {klo, lo[1], lo[2]}, zhi[3] = {khi, hi[1], hi[2]};
+    int64_t zlo[3] = {klo, lo[1], A.lo[2]}, zhi[3] = {khi, hi[1], hi[2]};
     geometry(p, k, batch, klo, khi, zlo, zhi, L);
     A.tiles_x = L.tiles_x;
     A.tiles_y = L.tiles_y;

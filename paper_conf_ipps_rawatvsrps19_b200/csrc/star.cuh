@@ -215,7 +215,9 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
                 const int gj = y0 + cy + py;
                 if (gj < a.hi[1] && col_in) {
                     double *o = a.out[0] + ((zbase + k) * a.ny + gj) * a.nx + gi;
-                    if (gi + 1 < a.hi[2]) {
+                    if (gi < a.xmin) {  // tile origin rounded down to even: first column is ring
+                        __stcs(o + 1, acc[py][1]);
+                    } else if (gi + 1 < a.hi[2]) {
                         if ((reinterpret_cast<uintptr_t>(o) & 15) == 0)
                             __stcs(reinterpret_cast<double2 *>(o), make_double2(acc[py][0], acc[py][1]));
                         else {

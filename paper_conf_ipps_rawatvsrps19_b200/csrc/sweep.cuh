@@ -53,6 +53,7 @@ struct SweepArgs {
     int64_t a1d_bstride[MAX1D];   // batch stride of each 1D array (0 = shared)
     int32_t lo[3], hi[3];         // output point range per axis (z, y, x)
     int32_t tiles_x, tiles_y, nchunk, zchunk;
+    int32_t xmin;                 // first interior x (lo[2] may be rounded down to even as tile origin)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -220,6 +221,12 @@ __global__ void __launch_bounds__(Geo<B, TX, TY, UX, UY, PF>::THREADS)
 
     int soff[2 * RZ + 1];
 
+    // the first window also needs planes kb-RZ .. kb+RZ-1 (the loop waits only
+    // for the newest plane of each window)
+    if constexpr (USE_TMA) {
+        for (int p = p0; p < kb + RZ && p <= plast; p++) mbar_wait(&bars[(p - p0) % NS], ((p - p0) / NS) & 1);
+    }
+
     for (int k = kb; k < ke; k++) {
         // prefetch plane k+RZ+PF into the slot of plane k-RZ-1 (freed by the
         // barrier that ended the previous iteration)
@@ -246,7 +253,7 @@ __global__ void __launch_bounds__(Geo<B, TX, TY, UX, UY, PF>::THREADS)
             for (int px = 0; px < UX; px++) {
                 const int ty = ly * UY + py, tx = lx * UX + px;
                 const int gj = y0 + ty, gi = x0 + tx;
-                const bool inside = gj < a.hi[1] && gi < a.hi[2];
+                const bool inside = gj < a.hi[1] && gi < a.hi[2] && gi >= a.xmin;
                 Tap<B, PX, NIN, SLOT> g;
                 g.ring = ring;
                 g.soff = soff;
