@@ -40,15 +40,15 @@ KernelDesc make_desc(const char *dag, int prio) {
 }
 
 // star-stencil kernel (star.cuh): 2-wide x patch, UY-tall y patch, register z-queue
-template <class B, int TX, int TY, int UY, int PF, bool TMA>
+template <class B, int TX, int TY, int UY, int PF, bool TMA, int QMODE = 0>
 KernelDesc make_star_desc(const char *dag, int prio) {
     using G = dev::StarGeo<B, TX, TY, UY, PF>;
     KernelDesc d;
     d.dag = dag;
     char buf[96];
-    std::snprintf(buf, sizeof buf, "star_%s_%dx%d_u2x%d_pf%d", TMA ? "tma" : "lsu", TX, TY, UY, PF);
+    std::snprintf(buf, sizeof buf, "star%s_%s_%dx%d_u2x%d_pf%d", QMODE ? "q" : "", TMA ? "tma" : "lsu", TX, TY, UY, PF);
     d.variant = buf;
-    d.fn = reinterpret_cast<const void *>(&dev::sdag_star<B, TX, TY, UY, PF, TMA>);
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_star<B, TX, TY, UY, PF, TMA, QMODE>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = TX;
@@ -66,6 +66,10 @@ KernelDesc make_star_desc(const char *dag, int prio) {
     d.prio = prio;
     return d;
 }
+
+// phase-unrolled queue (QMODE 1), TMA only
+#define SDAG_STARQ(v, BODY, DAG, TX, TY, UY, PF, PRIO) \
+    v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, 1>(DAG, PRIO))
 
 #define SDAG_STAR_PAIR(v, BODY, DAG, TX, TY, UY, PF, PRIO)                                \
     do {                                                                                   \

@@ -9,17 +9,26 @@
 //    (serial streaming with register reuse along the streamed dimension,
 //    P:611-638; the retiming idea of P:790-830 applied to the centre column),
 //  * a 2-wide x patch read with 128-bit LDS (blocked unrolling):
-//    each row window [x-R, x+2+R) is (R+1) aligned double2 loads,
+//    each row window [x-R, x+2+R) is a few aligned double2 loads,
 //  * a UY-tall y patch whose column [y-R, y+UY+R) is read once per plane,
 // so each point costs ~9 doubles of smem reads for R=4 (4.5 for R=1).
 // Planes arrive by TMA (cp.async.bulk.tensor.3d + mbarrier expect_tx) into a
 // ring of R+1+PF slots: plane p is used first as the queue head (its centre
 // values) and last, R iterations later, as the centre plane with its xy halo.
+// Slots are recycled through per-slot "empty" mbarriers (one arrival per
+// warp) instead of a CTA-wide barrier per plane, so warps do not wait for one
+// another; only the TMA-issuing thread waits for a slot to drain.
+//
+// QMODE 0: the queue is shifted with register moves after every plane;
+// QMODE 1: the plane loop is dispatched to NQ phase copies so the queue
+// rotates by compile-time indexing (no moves, NQ x the code).
 //
 // Arithmetic is re-associated relative to the spec (y/z taps first, then x,
 // then the centre, each group as fma(c_r, sum, acc)); parity is by the scaled
 // error gate (reading R13).
 #pragma once
+
+#include <type_traits>
 
 #include "sweep.cuh"
 
@@ -53,10 +62,23 @@ struct Jacobi7Star {
     }
 };
 
+// compile-time loop: f(std::integral_constant<int, 0>) ... f(<N-1>)
+template <int I, int N, class F>
+__device__ __forceinline__ void static_for_impl(F &&f) {
+    if constexpr (I < N) {
+        f(std::integral_constant<int, I>{});
+        static_for_impl<I + 1, N>(f);
+    }
+}
+template <int N, class F>
+__device__ __forceinline__ void static_for(F &&f) {
+    static_for_impl<0, N>(f);
+}
+
 template <class B, int TX, int TY, int UY, int PF>
 struct StarGeo {
     static constexpr int R = B::R;
-    static constexpr int NTX = TX / 2, NTY = TY / UY, THREADS = NTX * NTY;
+    static constexpr int NTX = TX / 2, NTY = TY / UY, THREADS = NTX * NTY, NWARPS = (THREADS + 31) / 32;
     // left/right box margin ML = R rounded up to even, so the centre column
     // cx + ML and the aligned x-window start cx are both 16-B aligned in smem
     static constexpr int ML = R + (R % 2);
@@ -65,12 +87,12 @@ struct StarGeo {
     static constexpr int PLANE_AL = ((PLANE * 8 + 127) / 128) * 128 / 8;
     static constexpr int NS = R + 1 + PF;  // ring slots
     static constexpr int NQ = 2 * R + 1;   // register queue depth
-    static constexpr int SMEM = NS * PLANE_AL * 8 + NS * 8;
+    static constexpr int SMEM = NS * PLANE_AL * 8 + 2 * NS * 8;  // ring + full/empty mbarriers
     static_assert(TX % 2 == 0 && TY % UY == 0, "tile");
     static_assert(PX <= 256 && PY <= 256, "TMA box");
 };
 
-template <class B, int TX, int TY, int UY, int PF, bool USE_TMA>
+template <class B, int TX, int TY, int UY, int PF, bool USE_TMA, int QMODE = 0>
 __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
     sdag_star(const __grid_constant__ SweepArgs a) {
     using G = StarGeo<B, TX, TY, UY, PF>;
@@ -78,7 +100,8 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
     double *ring = reinterpret_cast<double *>(smem_raw);
-    uint64_t *bars = reinterpret_cast<uint64_t *>(smem_raw + NS * PAL * 8);
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * PAL * 8);
+    uint64_t *empty = full + NS;
 
     const int tile_x = blockIdx.x, tile_y = blockIdx.y;
     const int chunk = blockIdx.z % a.nchunk;
@@ -92,16 +115,19 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
 
     const int t = threadIdx.x;
     const int lx = t % G::NTX, ly = t / G::NTX;
-    const int cx = 2 * lx;       // patch x offset inside the tile (even: 16-B aligned in smem)
-    const int cy = UY * ly;      // patch y offset inside the tile
+    const int cx = 2 * lx;   // patch x offset inside the tile (even: 16-B aligned in smem)
+    const int cy = UY * ly;  // patch y offset inside the tile
 
     auto issue = [&](int p) {
         const int slot = (p - p0) % NS;
         double *dst = ring + slot * PAL;
         if constexpr (USE_TMA) {
             if (t == 0) {
-                mbar_expect_tx(&bars[slot], uint32_t(G::PLANE * 8));
-                tma_load_3d(dst, &a.tmap[0], &bars[slot], x0 - ML, y0 - R, int(zbase + p));
+                // the previous occupant, plane p-NS, must have been released by every warp
+                const int prev = p - NS;
+                if (prev >= p0) mbar_wait(&empty[slot], ((prev - p0) / NS) & 1);
+                mbar_expect_tx(&full[slot], uint32_t(G::PLANE * 8));
+                tma_load_3d(dst, &a.tmap[0], &full[slot], x0 - ML, y0 - R, int(zbase + p));
             }
         } else {
             const int64_t pl = (zbase + p) * a.ny * a.nx;
@@ -113,18 +139,21 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
             }
         }
     };
-    auto wait = [&](int p) {
+    auto release = [&](int p) {  // every warp is done with plane p's slot
         if constexpr (USE_TMA) {
-            mbar_wait(&bars[(p - p0) % NS], ((p - p0) / NS) & 1);
-        } else {
-            cp_async_wait<PF>();
-            __syncthreads();
+            __syncwarp();
+            if ((t & 31) == 0)
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[(p - p0) % NS]))
+                             : "memory");
         }
     };
 
     if constexpr (USE_TMA) {
         if (t == 0) {
-            for (int s = 0; s < NS; s++) mbar_init(&bars[s], 1);
+            for (int s = 0; s < NS; s++) {
+                mbar_init(&full[s], 1);
+                mbar_init(&empty[s], G::NWARPS);
+            }
             asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         }
         __syncthreads();
@@ -134,35 +163,35 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
         if constexpr (!USE_TMA) cp_async_commit();
     }
 
-    double q[NQ][UY][2];  // q[d] = centre values of plane p-2R+d (d = 2R: newest)
-#pragma unroll
-    for (int d = 0; d < NQ; d++)
-#pragma unroll
-        for (int py = 0; py < UY; py++) q[d][py][0] = q[d][py][1] = 0.0;
+    // per-thread store geometry (fixed for the whole z-stream)
+    const int gi = x0 + cx;
+    const bool ok0 = gi >= a.xmin && gi < a.hi[2];
+    const bool ok1 = gi + 1 >= a.xmin && gi + 1 < a.hi[2];
+    const bool vec = ok0 && ok1 && (a.nx % 2 == 0) && ((reinterpret_cast<uintptr_t>(a.out[0]) & 15) == 0);
+    const int nrows = min(UY, a.hi[1] - (y0 + cy));
 
-    const bool col_in = (x0 + cx) < a.hi[2];
-    for (int p = p0; p <= plast; p++) {
+    double q[NQ][UY][2];  // register z-queue (see QMODE)
+
+    auto step = [&](auto phase, int p) {
+        constexpr int PH = decltype(phase)::value;  // slot of plane p in q
         {
             const int pn = p + PF;
             if (pn <= plast) issue(pn);
             if constexpr (!USE_TMA) cp_async_commit();
         }
-        wait(p);
-        // shift the queue and load the head (plane p's centre values)
-#pragma unroll
-        for (int d = 0; d < NQ - 1; d++)
-#pragma unroll
-            for (int py = 0; py < UY; py++) {
-                q[d][py][0] = q[d + 1][py][0];
-                q[d][py][1] = q[d + 1][py][1];
-            }
-        {
+        if constexpr (USE_TMA) {
+            mbar_wait(&full[(p - p0) % NS], ((p - p0) / NS) & 1);
+        } else {
+            cp_async_wait<PF>();
+            __syncthreads();
+        }
+        {  // queue head: plane p's centre values
             const double *hp = ring + ((p - p0) % NS) * PAL + (cy + R) * PX + (cx + ML);
 #pragma unroll
             for (int py = 0; py < UY; py++) {
                 const double2 v = *reinterpret_cast<const double2 *>(hp + py * PX);
-                q[NQ - 1][py][0] = v.x;
-                q[NQ - 1][py][1] = v.y;
+                q[PH][py][0] = v.x;
+                q[PH][py][1] = v.y;
             }
         }
         const int k = p - R;
@@ -171,7 +200,7 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
             double acc[UY][2];
 #pragma unroll
             for (int py = 0; py < UY; py++) acc[py][0] = acc[py][1] = 0.0;
-            // y and z taps: column rows [cy-R, cy+UY+R) of plane k
+            // y and z taps: column rows [cy-R, cy+UY+R) of plane k; z from the queue
             {
                 double col[UY + 2 * R][2];
 #pragma unroll
@@ -185,9 +214,12 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
 #pragma unroll
                     for (int px = 0; px < 2; px++)
 #pragma unroll
-                        for (int r = 1; r <= R; r++)
-                            B::yz(acc[py][px], a, r,
-                                  (col[py + R + r][px] + col[py + R - r][px]) + (q[R + r][py][px] + q[R - r][py][px]));
+                        for (int r = 1; r <= R; r++) {
+                            // plane k+d (k = p-R) lives in slot (PH - R + d) mod NQ
+                            const double zp = q[(PH + NQ - R + r) % NQ][py][px];
+                            const double zm = q[(PH + NQ - R - r) % NQ][py][px];
+                            B::yz(acc[py][px], a, r, (col[py + R + r][px] + col[py + R - r][px]) + (zp + zm));
+                        }
             }
             // x taps: the row window [cx-R, cx+2+R) lies in the aligned span
             // [cx, cx+WN) of smem columns; w[ML + px + dx] is the tap (px, dx)
@@ -208,29 +240,45 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
                     acc[py][px] = B::finish(acc[py][px], a, w[ML + px]);
                 }
             }
-            // interior-only streaming stores (2-wide when both points are inside)
-            const int gi = x0 + cx;
+            release(k);  // last use of plane k (as centre)
+            // interior-only streaming stores (16-B vector stores when both points are inside)
+            double *o = a.out[0] + ((zbase + k) * a.ny + (y0 + cy)) * a.nx + gi;
 #pragma unroll
             for (int py = 0; py < UY; py++) {
-                const int gj = y0 + cy + py;
-                if (gj < a.hi[1] && col_in) {
-                    double *o = a.out[0] + ((zbase + k) * a.ny + gj) * a.nx + gi;
-                    if (gi < a.xmin) {  // tile origin rounded down to even: first column is ring
-                        __stcs(o + 1, acc[py][1]);
-                    } else if (gi + 1 < a.hi[2]) {
-                        if ((reinterpret_cast<uintptr_t>(o) & 15) == 0)
-                            __stcs(reinterpret_cast<double2 *>(o), make_double2(acc[py][0], acc[py][1]));
-                        else {
-                            __stcs(o, acc[py][0]);
-                            __stcs(o + 1, acc[py][1]);
-                        }
+                if (py < nrows) {
+                    if (vec) {
+                        __stcs(reinterpret_cast<double2 *>(o), make_double2(acc[py][0], acc[py][1]));
                     } else {
-                        __stcs(o, acc[py][0]);
+                        if (ok0) __stcs(o, acc[py][0]);
+                        if (ok1) __stcs(o + 1, acc[py][1]);
                     }
                 }
+                o += a.nx;
             }
+        } else if (p < kb) {
+            release(p);  // a head-only plane (never a centre) is done
         }
-        __syncthreads();  // slot of plane k is reused by the next issue
+        if constexpr (!USE_TMA) __syncthreads();  // the LSU ring has no empty barriers
+    };
+
+    if constexpr (QMODE == 0) {
+        for (int p = p0; p <= plast; p++) {
+            step(std::integral_constant<int, NQ - 1>{}, p);
+#pragma unroll
+            for (int d = 0; d < NQ - 1; d++)
+#pragma unroll
+                for (int py = 0; py < UY; py++) {
+                    q[d][py][0] = q[d + 1][py][0];
+                    q[d][py][1] = q[d + 1][py][1];
+                }
+        }
+    } else {
+        for (int p = p0; p <= plast; p++) {
+            const int ph = (p - p0) % NQ;
+            static_for<NQ>([&](auto I) {
+                if (ph == decltype(I)::value) step(I, p);
+            });
+        }
     }
 }
 
