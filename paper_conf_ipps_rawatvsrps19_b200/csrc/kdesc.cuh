@@ -5,6 +5,7 @@
 
 #include "bodies.cuh"
 #include "kernels.hpp"
+#include "box27.cuh"
 #include "star.cuh"
 #include "sweep.cuh"
 
@@ -66,6 +67,40 @@ KernelDesc make_star_desc(const char *dag, int prio) {
     d.prio = prio;
     return d;
 }
+
+// 27-point box kernel (box27.cuh): retimed, folded in-plane partial sums
+template <int TX, int TY, int UY, int PF, bool TMA>
+KernelDesc make_box27_desc(const char *dag, int prio) {
+    using G = dev::BoxGeo<TX, TY, UY, PF>;
+    KernelDesc d;
+    d.dag = dag;
+    char buf[96];
+    std::snprintf(buf, sizeof buf, "box_%s_%dx%d_u2x%d_pf%d", TMA ? "tma" : "lsu", TX, TY, UY, PF);
+    d.variant = buf;
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_box27<TX, TY, UY, PF, TMA>);
+    d.threads = G::THREADS;
+    d.smem = G::SMEM;
+    d.tx = TX;
+    d.ty = TY;
+    d.ux = 2;
+    d.uy = UY;
+    d.pf = PF;
+    d.tma = TMA;
+    d.nin = 1;
+    d.nout = 1;
+    d.rz = 1;
+    d.ry = 1;
+    d.rx = G::ML;
+    d.rzr = 0;  // each plane is read once
+    d.prio = prio;
+    return d;
+}
+
+#define SDAG_BOX_PAIR(v, DAG, TX, TY, UY, PF, PRIO)                                 \
+    do {                                                                            \
+        v.push_back(make_box27_desc<TX, TY, UY, PF, true>(DAG, PRIO));              \
+        v.push_back(make_box27_desc<TX, TY, UY, PF, false>(DAG, PRIO + 100));       \
+    } while (0)
 
 // phase-unrolled queue (QMODE 1), TMA only
 #define SDAG_STARQ(v, BODY, DAG, TX, TY, UY, PF, PRIO) \
