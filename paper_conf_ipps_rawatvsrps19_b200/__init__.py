@@ -74,7 +74,13 @@ def _opts(order=-1, device=None, tune=False, batch=1, variant=None):
     if device == "none":
         o.device = SDAG_DEVICE_NONE
     elif device is None:
+        # libsdag links its own (static) CUDA runtime, whose "current device" is
+        # independent of torch's: bind to the device torch is using.
         o.device = SDAG_DEVICE_CURRENT
+        import sys
+        torch = sys.modules.get("torch")
+        if torch is not None and torch.cuda.is_available():
+            o.device = int(torch.cuda.current_device())
     else:
         o.device = int(device)
     o.tune = 1 if tune else 0

@@ -6,6 +6,7 @@
 #include "bodies.cuh"
 #include "kernels.hpp"
 #include "box27.cuh"
+#include "hyp.cuh"
 #include "star.cuh"
 #include "sweep.cuh"
 
@@ -100,6 +101,40 @@ KernelDesc make_box27_desc(const char *dag, int prio) {
     do {                                                                            \
         v.push_back(make_box27_desc<TX, TY, UY, PF, true>(DAG, PRIO));              \
         v.push_back(make_box27_desc<TX, TY, UY, PF, false>(DAG, PRIO + 100));       \
+    } while (0)
+
+// hypterm kernel (hyp.cuh): retimed z, folded fluxes, x-pairs
+template <int TX, int TY, int PF, bool TMA>
+KernelDesc make_hyp_desc(const char *dag, int prio) {
+    using G = dev::HypGeo<TX, TY, PF>;
+    KernelDesc d;
+    d.dag = dag;
+    char buf[96];
+    std::snprintf(buf, sizeof buf, "hyp_%s_%dx%d_u2x1_pf%d", TMA ? "tma" : "lsu", TX, TY, PF);
+    d.variant = buf;
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_hyp<TX, TY, PF, TMA>);
+    d.threads = G::THREADS;
+    d.smem = G::SMEM;
+    d.tx = TX;
+    d.ty = TY;
+    d.ux = 2;
+    d.uy = 1;
+    d.pf = PF;
+    d.tma = TMA;
+    d.nin = 8;
+    d.nout = 5;
+    d.rz = 4;
+    d.ry = 4;
+    d.rx = G::ML;
+    d.rzr = 4;  // z-halo planes streamed per chunk
+    d.prio = prio;
+    return d;
+}
+
+#define SDAG_HYP_PAIR(v, DAG, TX, TY, PF, PRIO)                                   \
+    do {                                                                          \
+        v.push_back(make_hyp_desc<TX, TY, PF, true>(DAG, PRIO));                  \
+        v.push_back(make_hyp_desc<TX, TY, PF, false>(DAG, PRIO + 100));           \
     } while (0)
 
 // phase-unrolled queue (QMODE 1), TMA only
