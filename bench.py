@@ -50,13 +50,16 @@ def load_peaks():
     return 6650.0, "fallback"
 
 
-def load_traffic(variant):
+def load_traffic(variant, dims, batch=1):
+    """DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum) from a
+    committed ncu --set full capture of this variant at this size, else None."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if not os.path.exists(p):
         return None
     with open(p) as f:
         d = json.load(f)
-    return d.get(variant)
+    key = variant + "@" + "x".join(str(x) for x in ([batch] if batch > 1 else []) + list(dims))
+    return d.get(key)
 
 
 class Clocks:
@@ -114,61 +117,135 @@ class Clocks:
 
 
 def cpu_baseline_lap25(A, c, seconds=10.0):
-    """Time the oracle (as it stands) on a bounded z-slab sample of the same input."""
+    """Time the oracle (as it stands) on the same 512^3 input: whole sweeps,
+    repeated for ~`seconds` of CPU work (the bounded sample)."""
     import oracle
     cores = len(os.sched_getaffinity(0))
     nz, ny, nx = A.shape
-    planes = 32
     out = np.zeros_like(A)
-    oracle.lap25(A, c, out=out, krange=(4, 4 + 2))  # warm (build + page-in)
+    oracle.lap25(A, c, out=out, krange=(4, 6))  # warm (build + page-in)
     reps, t0 = 0, time.perf_counter()
-    k0 = 4
     while True:
-        oracle.lap25(A, c, out=out, krange=(k0, k0 + planes))
+        oracle.lap25(A, c, out=out)
         reps += 1
-        k0 = 4 + (k0 + planes - 4) % (nz - 8 - planes)
         if time.perf_counter() - t0 >= seconds:
             break
     dt = time.perf_counter() - t0
-    pts = reps * planes * (ny - 8) * (nx - 8)
+    pts = reps * (nz - 8) * (ny - 8) * (nx - 8)
     return {"value": pts * 29 / dt / 1e9, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
-            "sample": f"{reps} x {planes}-plane z-slabs of the 512^3 input ({pts} interior points), "
-                      f"{dt:.1f} s, OpenMP over k"}
+            "sample": f"{reps} full 512^3 sweeps of the benchmark input ({pts} interior points), {dt:.1f} s, "
+                      f"OpenMP over k with {cores} threads"}
 
 
 def run_reference(args):
-    """--impl reference: the CPU oracle on the host cores, same metric/config."""
+    """--impl reference: the CPU oracle (this tier's reference arm) on the host
+    cores, same metric and config: each step is one full 512^3 sweep of the same
+    seeded input (~0.1-0.3 s of CPU work per step)."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
     import synth
     dims = CONFIGS["lap25"][1]
-    ins, sc = synth.lap25_inputs(dims)
+    ins, sc = synth.lap25_inputs(dims, cfg="cfg2")
     A = ins["A"]
     c = [sc[k] for k in ("c0", "c1", "c2", "c3", "c4")]
     import oracle
     cores = len(os.sched_getaffinity(0))
     out = np.zeros_like(A)
-    planes = 16
     nz, ny, nx = dims
     oracle.lap25(A, c, out=out, krange=(4, 6))
     for _ in range(args.warmup):
-        oracle.lap25(A, c, out=out, krange=(4, 4 + planes))
+        oracle.lap25(A, c, out=out)
     t0 = time.perf_counter()
-    for s in range(args.steps):
-        k0 = 4 + (s * planes) % (nz - 8 - planes)
-        oracle.lap25(A, c, out=out, krange=(k0, k0 + planes))
+    for _ in range(args.steps):
+        oracle.lap25(A, c, out=out)
     dt = time.perf_counter() - t0
-    pts = args.steps * planes * (ny - 8) * (nx - 8)
+    pts = args.steps * (nz - 8) * (ny - 8) * (nx - 8)
     val = pts * 29 / dt / 1e9
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "GFLOP/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": CONFIGS["lap25"][2], "stencil": "lap25", "grid": list(dims),
-                       "step": f"oracle sweep of a {planes}-plane z-slab sample (bounded CPU time)"},
+                       "step": "one full oracle sweep of the 512^3 input on the host cores"},
             "cpu_baseline": {"value": val, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
-                             "sample": f"{args.steps} steps x {planes} planes x {ny - 8}x{nx - 8} interior points"},
+                             "sample": f"{args.steps} full 512^3 sweeps (all interior points)"},
             "e2e": {"value": val, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+    return 0
+
+
+def run_other(args):
+    """One line for another BASELINE stencil at N=1 (recorded under profiles/, not the headline).
+    Inputs: seeded torch generator on the device (timing is data-independent; parity of
+    the same kernels on synth/ inputs is in tests/test_gpu_parity.py)."""
+    import torch
+    import paper_conf_ipps_rawatvsrps19_b200 as sdag
+    name = args.config
+    spec = sdag.spec_text(name)
+    dims = CONFIGS[name][1]
+    torch.cuda.set_device(0)
+    g = torch.Generator(device="cuda").manual_seed(20190520)
+    batch, T = 1, 1
+    if name == "jacobi7":
+        batch = 128  # config 1b: 128 independent 64^3 problems in one launch (latency-bound alone)
+    plan = sdag.Plan(spec, dims, batch=batch, tune=args.tune, variant=args.variant)
+    info = plan.info
+    shape = (batch, *dims) if batch > 1 else dims
+    scal = {"jacobi7": [4.0, 0.5, 0.25], "hypterm": [0.5, 0.25, 0.125, 0.8, -0.2, 4 / 105, -1 / 280],
+            "rhs4center": [0.75, 1 / 6, 1 / 144, 1.0, 1.0], "smooth27": [-128 / 30, 14 / 30, 3 / 30, 1 / 30, 0.125]}[name]
+    arrs = [torch.rand(shape, dtype=torch.float64, device="cuda", generator=g) + 0.5
+            for _ in range(info["n_arrays3d"])]
+    a1 = [torch.rand(dims[2 - q], dtype=torch.float64, device="cuda", generator=g) + 0.5
+          for q in range(info["n_arrays1d"])]
+    if name == "smooth27":
+        T = 12  # config 5: iterated T = 12 sweeps (Table I "T", reading R5)
+        b0, b1 = arrs[1], arrs[0]
+
+        def step():
+            plan.apply_iterated(b0, b1, T, scal)
+    elif batch > 1:
+        def step():
+            plan.apply_batched(batch, arrs, a1, scal)
+    else:
+        def step():
+            plan.apply(arrs, a1, scal)
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    l0 = sdag.launch_count()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with Clocks(0) as clk:
+        torch.cuda.synchronize()
+        e0.record()
+        for _ in range(args.steps):
+            step()
+        e1.record()
+        torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / args.steps
+    launches = sdag.launch_count() - l0
+    pts = info["points"] * batch * T
+    flops = info["flops_per_point"] * pts
+    byts = info["bytes_per_point"] * pts
+    kms = ms / (launches / args.steps)
+    hbm, src = load_peaks()
+    if name == "rhs4center":
+        fp64 = sdag.fp64_peak()
+        achieved = info["flops_per_point"] * info["points"] / (kms * 1e-3) / 1e12
+        roof = {"bound": "fp64", "achieved": achieved, "peak": fp64 / 1e12, "unit": "TFLOP/s", "frac": achieved * 1e12 / fp64,
+                "peak_source": "measured DFMA micro-benchmark (sdag_measure_fp64_peak) in this run"}
+    else:
+        achieved = info["bytes_per_point"] * info["points"] * batch / (kms * 1e-3) / 1e9
+        roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
+                "peak_source": src}
+    roof.update({"traffic": load_traffic(info["variant"], dims, batch), "kernel_ms": kms, "kernel": info["variant"]})
+    line = {"metric": METRIC, "value": flops / (ms * 1e-3) / 1e9, "unit": "GFLOP/s", "n_gpus": 1,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded torch generator)",
+            "config": {"workload": CONFIGS[name][2], "stencil": name, "grid": list(dims), "batch": batch,
+                       "sweeps_per_step": T, "variant": info["variant"], "flops_per_point": info["flops_per_point"],
+                       "bytes_per_point": info["bytes_per_point"]},
+            "hbm_gbs": byts / (ms * 1e-3) / 1e9, "roofline": roof, "gpu_launches": launches,
+            "clocks": clk.summary()}
     print(json.dumps(line))
     return 0
 
@@ -183,10 +260,14 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--variant", default=None)
     ap.add_argument("--tune", action="store_true")
+    ap.add_argument("--config", default="lap25", choices=list(CONFIGS),
+                    help="lap25 = the headline line; the others record the remaining BASELINE stencils (N=1)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
         return run_reference(args)
+    if args.config != "lap25":
+        return run_other(args)
 
     import torch
     import paper_conf_ipps_rawatvsrps19_b200 as sdag
@@ -282,7 +363,7 @@ def main():
     peak, peak_src = load_peaks()
     bytes_launch = info["bytes_per_point"] * info["points"]
     achieved = bytes_launch / (kms * 1e-3) / 1e9
-    traffic = load_traffic(info["variant"])
+    traffic = load_traffic(info["variant"], ldims) if world == 1 else None
 
     e2e = None
     if not args.no_e2e and world == 1:

@@ -289,6 +289,7 @@ void dist_apply(Dist *d, double *const *a3, int n3, const double *const *a1, int
     if (p->kernel().tma)
         for (int f = 0; f < n3; f++)
             if (reinterpret_cast<uintptr_t>(a3[f]) % 16) throw Error(SDAG_ERR_INVALID_ARG, "grid arrays must be 16-B aligned");
+    check_cuda(cudaSetDevice(p->device), "cudaSetDevice");  // libsdag's runtime: bind the plan's device
     sweep_split(d, a3, a1, s, compute, comm_stream(d, comm), true);
 }
 
@@ -302,6 +303,7 @@ void dist_apply_iterated(Dist *d, double *b0, double *b1, int T, const double *s
     if (ns != p->ns() || !b0 || !b1 || b0 == b1) throw Error(SDAG_ERR_INVALID_ARG, "bad arguments");
     int fin = -1, fout = -1;
     for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
+    check_cuda(cudaSetDevice(p->device), "cudaSetDevice");
     cudaStream_t cs = comm_stream(d, comm);
     double *bufs[2] = {b0, b1};
     for (int t = 0; t < T; t++) {
@@ -324,6 +326,7 @@ void dist_apply_iterated_loopback(Dist **ds, int n, double *const *b0, double *c
         throw Error(SDAG_ERR_INVALID_ARG, "iterated loopback needs a 1-input 1-output plan");
     int fin = -1, fout = -1;
     for (int f = 0; f < 2; f++) (p0->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
+    check_cuda(cudaSetDevice(p0->device), "cudaSetDevice");
     const int64_t rz = ds[0]->rz;
     const size_t plane = size_t(p0->dims[1] * p0->dims[2]);
     for (int t = 0; t < T; t++) {

@@ -1,14 +1,14 @@
 // Instantiations for the 27-point smoother: the retimed/folded box kernel
 // first, the generic skeleton as fallback variants.
+// Order = heuristic preference, from tools/perf_sweep.py on B200 at 512^3.
 #include "kdesc.cuh"
 namespace sdag {
 void add_kernels_smooth27(std::vector<KernelDesc> &v) {
-    SDAG_BOX_PAIR(v, "smooth27", 64, 16, 4, 3, 0);
-    SDAG_BOX_PAIR(v, "smooth27", 32, 32, 4, 3, 1);
-    SDAG_BOX_PAIR(v, "smooth27", 64, 32, 4, 3, 2);
-    SDAG_BOX_PAIR(v, "smooth27", 64, 16, 2, 3, 3);
-    SDAG_BOX_PAIR(v, "smooth27", 128, 16, 4, 2, 4);
+    SDAG_BOX_PAIR(v, "smooth27", 128, 16, 4, 2, 0);
+    SDAG_BOX_PAIR(v, "smooth27", 64, 32, 4, 3, 1);
+    SDAG_BOX_PAIR(v, "smooth27", 64, 16, 4, 3, 2);
+    SDAG_BOX_PAIR(v, "smooth27", 128, 16, 4, 3, 3);
+    SDAG_BOX_PAIR(v, "smooth27", 128, 32, 4, 2, 4);
     SDAG_PAIR(v, Smooth27, "smooth27", 64, 16, 1, 4, 2, 10);
-    SDAG_PAIR(v, Smooth27, "smooth27", 32, 16, 1, 2, 2, 11);
 }
 }  // namespace sdag

@@ -64,7 +64,7 @@ if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("report")
     ap.add_argument("out")
-    ap.add_argument("--variant")
+    ap.add_argument("--variant", help="traffic key: VARIANT@[batchx]NZxNYxNX")
     ap.add_argument("--alg-bytes", type=float)
     ap.add_argument("--flops", type=float)
     a = ap.parse_args()
