@@ -51,6 +51,48 @@ def uniform(shape, lo: float, hi: float, *key, seed: int = MASTER_SEED, chunk: i
     return out.reshape(shape)
 
 
+def uniform_at(lin_index, lo: float, hi: float, *key, seed: int = MASTER_SEED) -> np.ndarray:
+    """The elements of uniform(shape, lo, hi, *key) at the given C-order linear
+    indices (counter-based: no need to generate the whole array)."""
+    idx = np.asarray(lin_index, dtype=np.uint64)
+    base = np.uint64((seed ^ key_hash(*key)) & 0xFFFFFFFFFFFFFFFF)
+    with np.errstate(over="ignore"):
+        z = splitmix64(idx + base) >> np.uint64(11)
+    return z.astype(np.float64) * ((hi - lo) * 2.0 ** -53) + lo
+
+
+def uniform_torch(shape, lo: float, hi: float, *key, seed: int = MASTER_SEED, device="cuda", chunk: int = 1 << 26):
+    """Same values as uniform(), generated on a torch device (for grids too large
+    to build on the host).  int64 two's-complement arithmetic reproduces the
+    uint64 splitmix64 bit for bit (logical shifts are masked)."""
+    import torch
+
+    n = int(np.prod(shape))
+    base = (seed ^ key_hash(*key)) & 0xFFFFFFFFFFFFFFFF
+
+    def s64(v):  # uint64 constant -> int64 bit pattern
+        return v - (1 << 64) if v >= (1 << 63) else v
+
+    m1, m2, gold = s64(0xBF58476D1CE4E5B9), s64(0x94D049BB133111EB), s64(0x9E3779B97F4A7C15)
+
+    def lsr(x, s):
+        return (x >> s) & ((1 << (64 - s)) - 1)
+
+    out = torch.empty(n, dtype=torch.float64, device=device)
+    scale = (hi - lo) * 2.0 ** -53
+    for s0 in range(0, n, chunk):
+        e = min(n, s0 + chunk)
+        z = torch.arange(s0, e, dtype=torch.int64, device=device)
+        z = z + s64(base)
+        z = z + gold
+        z = (z ^ lsr(z, 30)) * m1
+        z = (z ^ lsr(z, 27)) * m2
+        z = z ^ lsr(z, 31)
+        z = lsr(z, 11)
+        out[s0:e] = z.to(torch.float64) * scale + lo
+    return out.view(*shape)
+
+
 def integers(shape, lo: int, hi: int, *key, seed: int = MASTER_SEED) -> np.ndarray:
     """Uniform integers in [lo, hi) as float64 (exact), keyed like uniform()."""
     n = int(np.prod(shape))
