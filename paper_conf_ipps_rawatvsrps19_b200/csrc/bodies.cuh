@@ -212,5 +212,18 @@ struct J1d3pt : BodyBase {
     }
 };
 
+// Trivial-fission wrapper (Fig 3b): evaluate only output M of
+// body B; the other outputs and every temporary they alone need are dead code.
+template <class B, int M>
+struct OnlyOut : B {
+    static constexpr int NOUT = 1;
+    template <class G>
+    __device__ __forceinline__ static void eval(const G &g, double (&o)[1]) {
+        double all[B::NOUT];
+        B::eval(g, all);
+        o[0] = all[M];
+    }
+};
+
 }  // namespace dev
 }  // namespace sdag

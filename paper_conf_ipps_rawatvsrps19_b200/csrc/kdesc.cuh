@@ -2,6 +2,7 @@
 #pragma once
 
 #include <cstdio>
+#include <utility>
 
 #include "bodies.cuh"
 #include "kernels.hpp"
@@ -145,6 +146,26 @@ KernelDesc make_hyp_desc(const char *dag, int prio) {
     do {                                                                                   \
         v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true>(DAG, PRIO));           \
         v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, false>(DAG, PRIO + 100));    \
+    } while (0)
+
+// trivial-fission variant of the generic skeleton: NOUT kernels, kernel m
+// evaluating OnlyOut<B, m> (named "fis_...")
+template <class B, int TX, int TY, int UX, int UY, int PF, bool TMA, int... M>
+KernelDesc make_fission_desc(const char *dag, int prio, std::integer_sequence<int, M...>) {
+    KernelDesc d = make_desc<B, TX, TY, UX, UY, PF, TMA>(dag, prio);
+    d.variant = "fis_" + d.variant;
+    d.fission = true;
+    d.fission_fns = {reinterpret_cast<const void *>(&dev::sdag_sweep<dev::OnlyOut<B, M>, TX, TY, UX, UY, PF, TMA>)...};
+    d.fn = d.fission_fns[0];
+    return d;
+}
+
+#define SDAG_FISSION_PAIR(v, BODY, DAG, TX, TY, UX, UY, PF, PRIO)                                                \
+    do {                                                                                                       \
+        v.push_back(make_fission_desc<dev::BODY, TX, TY, UX, UY, PF, true>(                                   \
+            DAG, PRIO, std::make_integer_sequence<int, dev::BODY::NOUT>{}));                                   \
+        v.push_back(make_fission_desc<dev::BODY, TX, TY, UX, UY, PF, false>(                                  \
+            DAG, PRIO + 100, std::make_integer_sequence<int, dev::BODY::NOUT>{}));                             \
     } while (0)
 
 // a TMA variant and its LSU twin (same geometry) for unaligned grids

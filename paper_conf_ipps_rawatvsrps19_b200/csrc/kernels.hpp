@@ -10,6 +10,8 @@ struct KernelDesc {
     std::string dag;      // registry DAG this kernel evaluates
     std::string variant;  // "tma_64x16_u1x4_pf2", ...
     const void *fn = nullptr;
+    bool fission = false;                 // trivial fission: one launch per output
+    std::vector<const void *> fission_fns;  // fission kernel for output m
     int threads = 0, smem = 0;
     int tx = 0, ty = 0, ux = 0, uy = 0, pf = 0;
     bool tma = false;

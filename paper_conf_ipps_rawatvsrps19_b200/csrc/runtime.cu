@@ -232,20 +232,31 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *
 
     static std::mutex attr_mu;
     static std::map<const void *, int> attr_done;
-    {
-        std::lock_guard<std::mutex> g(attr_mu);
-        int &d = attr_done[k.fn];
-        if (d < k.smem) {
-            check_cuda(cudaFuncSetAttribute(k.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, k.smem),
-                       "cudaFuncSetAttribute(max dynamic smem)");
-            d = k.smem;
+    // trivial-fission variants (Fig 3): one kernel per output,
+    // each evaluating only that output (shared temporaries replicated)
+    const int nlaunch = k.fission ? int(k.fission_fns.size()) : 1;
+    for (int q = 0; q < nlaunch; q++) {
+        const void *fn = k.fission ? k.fission_fns[q] : k.fn;
+        {
+            std::lock_guard<std::mutex> g(attr_mu);
+            int &d = attr_done[fn];
+            if (d < k.smem) {
+                check_cuda(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, k.smem),
+                           "cudaFuncSetAttribute(max dynamic smem)");
+                d = k.smem;
+            }
         }
+        dev::SweepArgs Aq = A;
+        if (k.fission) {
+            for (int m = 0; m < dev::MAXOUT; m++) Aq.out[m] = nullptr;
+            Aq.out[0] = A.out[q];
+        }
+        dim3 grid(L.tiles_x, L.tiles_y, L.nchunk * batch);
+        if (grid.z > 65535 || grid.y > 65535) throw Error(SDAG_ERR_DOMAIN, "grid too large (batch x chunks > 65535)");
+        void *args[] = {&Aq};
+        check_cuda(cudaLaunchKernel(fn, grid, dim3(k.threads), args, size_t(k.smem), stream), "sweep launch");
+        count_launch();
     }
-    dim3 grid(L.tiles_x, L.tiles_y, L.nchunk * batch);
-    if (grid.z > 65535 || grid.y > 65535) throw Error(SDAG_ERR_DOMAIN, "grid too large (batch x chunks > 65535)");
-    void *args[] = {&A};
-    check_cuda(cudaLaunchKernel(k.fn, grid, dim3(k.threads), args, size_t(k.smem), stream), "sweep launch");
-    count_launch();
 }
 
 static void validate_arrays(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, int ns,
@@ -564,7 +575,7 @@ void plan_fill_info(Plan *p, sdag_plan_info *info) {
     info->flops_per_point = p->an.flops_per_point;
     info->bytes_per_point = p->bytes_per_point();
     info->oi_paper = p->an.n_io_arrays ? p->an.flops_per_point / (8.0 * p->an.n_io_arrays) : 0.0;
-    info->n_kernels = 1;
+    info->n_kernels = (!p->cands.empty() && p->kernel().fission) ? int(p->kernel().fission_fns.size()) : 1;
     info->n_variants = int(p->cands.size());
     info->dag = p->reg ? p->reg->name.c_str() : "";
     info->variant = p->cands.empty() ? "" : p->kernel().variant.c_str();
