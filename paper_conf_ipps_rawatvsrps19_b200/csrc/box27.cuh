@@ -41,7 +41,12 @@ struct BoxGeo {
     static_assert(PX <= 256 && PY <= 256, "TMA box");
 };
 
-template <int TX, int TY, int UY, int PF, bool USE_TMA>
+// FORM 0: the 27-point smoother (scalars w0..w3, nu).
+// FORM 1: Listing 1's 7-point Jacobi (scalars h2inv, a, b) in the same
+//   retimed form: T_k = s1_k - 6 s0_k + s0_{k-1} is formed when plane k
+//   streams past and B[k] = a A[k] - (b h2inv)(T_k + s0_{k+1}) when plane k+1
+//   does (2 doubles of z-state per point).
+template <int TX, int TY, int UY, int PF, bool USE_TMA, int FORM = 0>
 __global__ void __launch_bounds__(BoxGeo<TX, TY, UY, PF>::THREADS)
     sdag_box27(const __grid_constant__ SweepArgs a) {
     using G = BoxGeo<TX, TY, UY, PF>;
@@ -103,6 +108,7 @@ __global__ void __launch_bounds__(BoxGeo<TX, TY, UY, PF>::THREADS)
     }
 
     const double w0 = a.s[0], w1 = a.s[1], w2 = a.s[2], w3 = a.s[3], nu = a.s[4];
+    const double ja = a.s[1], jc = a.s[2] * a.s[0];  // FORM 1: a, c = b*h2inv
     const int gi = x0 + cx;
     const bool ok0 = gi >= a.xmin && gi < a.hi[2];
     const bool ok1 = gi + 1 >= a.xmin && gi + 1 < a.hi[2];
@@ -157,12 +163,17 @@ __global__ void __launch_bounds__(BoxGeo<TX, TY, UY, PF>::THREADS)
                 const int c = ML + px;  // centre column in w
                 const double s0 = w[py + 1][c];
                 const double s1 = (w[py + 1][c - 1] + w[py + 1][c + 1]) + (w[py][c] + w[py + 2][c]);
-                const double s2 = (w[py][c - 1] + w[py][c + 1]) + (w[py + 2][c - 1] + w[py + 2][c + 1]);
-                const double cc = fma(w2, s2, fma(w1, s1, w0 * s0));
-                const double uu = fma(w3, s2, fma(w2, s1, w1 * s0));
-                res[px] = fma(nu, Tprev[py][px] + uu, Aprev[py][px]);  // B[k] = A[k] + nu(u_{k-1} + c_k + u_{k+1})
-                Tprev[py][px] = Uprev[py][px] + cc;                   // u_{p-1} + c_p
-                Uprev[py][px] = uu;
+                if constexpr (FORM == 0) {
+                    const double s2 = (w[py][c - 1] + w[py][c + 1]) + (w[py + 2][c - 1] + w[py + 2][c + 1]);
+                    const double cc = fma(w2, s2, fma(w1, s1, w0 * s0));
+                    const double uu = fma(w3, s2, fma(w2, s1, w1 * s0));
+                    res[px] = fma(nu, Tprev[py][px] + uu, Aprev[py][px]);  // B[k] = A[k] + nu(u_{k-1} + c_k + u_{k+1})
+                    Tprev[py][px] = Uprev[py][px] + cc;                   // u_{p-1} + c_p
+                    Uprev[py][px] = uu;
+                } else {
+                    res[px] = ja * Aprev[py][px] - jc * (Tprev[py][px] + s0);      // B[k], k = p-1
+                    Tprev[py][px] = fma(-6.0, s0, s1 + Aprev[py][px]);           // T_p
+                }
                 Aprev[py][px] = s0;
             }
             if (k >= kb && py < nrows) {

@@ -71,15 +71,16 @@ KernelDesc make_star_desc(const char *dag, int prio) {
 }
 
 // 27-point box kernel (box27.cuh): retimed, folded in-plane partial sums
-template <int TX, int TY, int UY, int PF, bool TMA>
+template <int TX, int TY, int UY, int PF, bool TMA, int FORM = 0>
 KernelDesc make_box27_desc(const char *dag, int prio) {
     using G = dev::BoxGeo<TX, TY, UY, PF>;
     KernelDesc d;
     d.dag = dag;
     char buf[96];
-    std::snprintf(buf, sizeof buf, "box_%s_%dx%d_u2x%d_pf%d", TMA ? "tma" : "lsu", TX, TY, UY, PF);
+    std::snprintf(buf, sizeof buf, "%s_%s_%dx%d_u2x%d_pf%d", FORM ? "cross" : "box", TMA ? "tma" : "lsu", TX, TY, UY,
+                  PF);
     d.variant = buf;
-    d.fn = reinterpret_cast<const void *>(&dev::sdag_box27<TX, TY, UY, PF, TMA>);
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_box27<TX, TY, UY, PF, TMA, FORM>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = TX;
@@ -97,6 +98,12 @@ KernelDesc make_box27_desc(const char *dag, int prio) {
     d.prio = prio;
     return d;
 }
+
+#define SDAG_CROSS_PAIR(v, DAG, TX, TY, UY, PF, PRIO)                               \
+    do {                                                                            \
+        v.push_back(make_box27_desc<TX, TY, UY, PF, true, 1>(DAG, PRIO));           \
+        v.push_back(make_box27_desc<TX, TY, UY, PF, false, 1>(DAG, PRIO + 100));    \
+    } while (0)
 
 #define SDAG_BOX_PAIR(v, DAG, TX, TY, UY, PF, PRIO)                                 \
     do {                                                                            \

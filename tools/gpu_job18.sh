@@ -1,0 +1,2 @@
+cd $GRAFT_REPO_ROOT
+timeout 900 python tools/perf_sweep.py jacobi7 > gpurun_out/perf_sweep.jsonl 2> gpurun_out/perf_sweep.err
