@@ -43,15 +43,16 @@ KernelDesc make_desc(const char *dag, int prio) {
 }
 
 // star-stencil kernel (star.cuh): 2-wide x patch, UY-tall y patch, register z-queue
-template <class B, int TX, int TY, int UY, int PF, bool TMA, int QMODE = 0>
+template <class B, int TX, int TY, int UY, int PF, bool TMA, int QMODE = 0, int MINB = 1>
 KernelDesc make_star_desc(const char *dag, int prio) {
     using G = dev::StarGeo<B, TX, TY, UY, PF>;
     KernelDesc d;
     d.dag = dag;
     char buf[96];
-    std::snprintf(buf, sizeof buf, "star%s_%s_%dx%d_u2x%d_pf%d", QMODE ? "q" : "", TMA ? "tma" : "lsu", TX, TY, UY, PF);
+    std::snprintf(buf, sizeof buf, "star%s_%s_%dx%d_u2x%d_pf%d%s", QMODE == 1 ? "q" : (QMODE == 2 ? "DIFFmem" : (QMODE == 3 ? "DIFFnost" : "")), TMA ? "tma" : "lsu", TX, TY, UY, PF,
+                  MINB > 1 ? (MINB == 2 ? "_mb2" : "_mb3") : "");
     d.variant = buf;
-    d.fn = reinterpret_cast<const void *>(&dev::sdag_star<B, TX, TY, UY, PF, TMA, QMODE>);
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_star<B, TX, TY, UY, PF, TMA, QMODE, MINB>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = TX;
@@ -144,6 +145,28 @@ KernelDesc make_hyp_desc(const char *dag, int prio) {
         v.push_back(make_hyp_desc<TX, TY, PF, true>(DAG, PRIO));                  \
         v.push_back(make_hyp_desc<TX, TY, PF, false>(DAG, PRIO + 100));           \
     } while (0)
+
+// register-capped variant: __launch_bounds__(threads, MINB), TMA only
+#define SDAG_STAR_MB(v, BODY, DAG, TX, TY, UY, PF, MB, PRIO) \
+    v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, 0, MB>(DAG, PRIO))
+
+// star2: z-taps k+1..k+R from the ring, k-1..k-R in a register queue
+template <class B, int TX, int TY, int UY, int PF, bool TMA, int MINB = 1>
+KernelDesc make_star2_desc(const char *dag, int prio) {
+    KernelDesc d = make_star_desc<B, TX, TY, UY, PF, TMA, 0, MINB>(dag, prio);
+    d.variant = "star2" + d.variant.substr(4);
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_star2<B, TX, TY, UY, PF, TMA, MINB>);
+    return d;
+}
+#define SDAG_STAR2_PAIR(v, BODY, DAG, TX, TY, UY, PF, MB, PRIO)                            \
+    do {                                                                                   \
+        v.push_back(make_star2_desc<dev::BODY, TX, TY, UY, PF, true, MB>(DAG, PRIO));      \
+        v.push_back(make_star2_desc<dev::BODY, TX, TY, UY, PF, false, MB>(DAG, PRIO + 100)); \
+    } while (0)
+
+// code-differencing variants: QMODE 2 = no arithmetic, 3 = no stores (profiling only)
+#define SDAG_STAR_DIFF(v, BODY, DAG, TX, TY, UY, PF, QM, PRIO) \
+    v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, QM, 1>(DAG, PRIO))
 
 // phase-unrolled queue (QMODE 1), TMA only
 #define SDAG_STARQ(v, BODY, DAG, TX, TY, UY, PF, PRIO) \

@@ -473,6 +473,9 @@ Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_pla
         if (k.dag != p->reg->name) continue;
         if (k.tma && p->dims[2] % 2 != 0) continue;
         if (k.smem > 227 * 1024) continue;
+        // code-differencing variants compute something else on purpose:
+        // only reachable through force_variant
+        if (k.prio >= 1000 && k.variant != p->force_variant) continue;
         p->cands.push_back(&k);
     }
     std::stable_sort(p->cands.begin(), p->cands.end(),

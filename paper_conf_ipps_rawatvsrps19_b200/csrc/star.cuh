@@ -92,8 +92,8 @@ struct StarGeo {
     static_assert(PX <= 256 && PY <= 256, "TMA box");
 };
 
-template <class B, int TX, int TY, int UY, int PF, bool USE_TMA, int QMODE = 0>
-__global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
+template <class B, int TX, int TY, int UY, int PF, bool USE_TMA, int QMODE = 0, int MINB = 1>
+__global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
     sdag_star(const __grid_constant__ SweepArgs a) {
     using G = StarGeo<B, TX, TY, UY, PF>;
     constexpr int R = G::R, PX = G::PX, NS = G::NS, NQ = G::NQ, PAL = G::PLANE_AL, ML = G::ML, WN = G::WN;
@@ -200,6 +200,11 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
             double acc[UY][2];
 #pragma unroll
             for (int py = 0; py < UY; py++) acc[py][0] = acc[py][1] = 0.0;
+            if constexpr (QMODE >= 2 && QMODE != 3) {
+                // code differencing: memory pipeline only, no stencil arithmetic
+#pragma unroll
+                for (int py = 0; py < UY; py++) acc[py][0] = q[PH][py][0], acc[py][1] = q[PH][py][1];
+            } else {
             // y and z taps: column rows [cy-R, cy+UY+R) of plane k; z from the queue
             {
                 double col[UY + 2 * R][2];
@@ -209,12 +214,13 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
                     col[r][0] = v.x;
                     col[r][1] = v.y;
                 }
+                // r outermost: 2*UY independent accumulation chains per step
 #pragma unroll
-                for (int py = 0; py < UY; py++)
+                for (int r = 1; r <= R; r++)
 #pragma unroll
-                    for (int px = 0; px < 2; px++)
+                    for (int py = 0; py < UY; py++)
 #pragma unroll
-                        for (int r = 1; r <= R; r++) {
+                        for (int px = 0; px < 2; px++) {
                             // plane k+d (k = p-R) lives in slot (PH - R + d) mod NQ
                             const double zp = q[(PH + NQ - R + r) % NQ][py][px];
                             const double zm = q[(PH + NQ - R - r) % NQ][py][px];
@@ -234,18 +240,20 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
                     w[2 * c + 1] = v.y;
                 }
 #pragma unroll
-                for (int px = 0; px < 2; px++) {
+                for (int r = 1; r <= R; r++)
 #pragma unroll
-                    for (int r = 1; r <= R; r++) B::x(acc[py][px], a, r, w[ML + px + r] + w[ML + px - r]);
-                    acc[py][px] = B::finish(acc[py][px], a, w[ML + px]);
-                }
+                    for (int px = 0; px < 2; px++) B::x(acc[py][px], a, r, w[ML + px + r] + w[ML + px - r]);
+#pragma unroll
+                for (int px = 0; px < 2; px++) acc[py][px] = B::finish(acc[py][px], a, w[ML + px]);
+            }
             }
             release(k);  // last use of plane k (as centre)
             // interior-only streaming stores (16-B vector stores when both points are inside)
             double *o = a.out[0] + ((zbase + k) * a.ny + (y0 + cy)) * a.nx + gi;
 #pragma unroll
             for (int py = 0; py < UY; py++) {
-                if (py < nrows) {
+                // QMODE 3 (code differencing): arithmetic kept alive, stores (almost) never issued
+                if (py < nrows && (QMODE != 3 || acc[py][0] == 12345.678)) {
                     if (vec) {
                         __stcs(reinterpret_cast<double2 *>(o), make_double2(acc[py][0], acc[py][1]));
                     } else {
@@ -279,6 +287,181 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, 1)
                 if (ph == decltype(I)::value) step(I, p);
             });
         }
+    }
+}
+
+
+// sdag_star2: same ring/patch design, but the z-taps k+1..k+R are read from the
+// ring (those planes are resident anyway: plane p = k+R is the newest) and only
+// k-1..k-R live in registers.  Halves the register queue (R instead of 2R+1
+// values per point) and its per-plane shifting, for ~3 more doubles of smem
+// reads per point (B200: the star kernel is issue-bound, not smem-bound).
+template <class B, int TX, int TY, int UY, int PF, bool USE_TMA, int MINB = 1>
+__global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
+    sdag_star2(const __grid_constant__ SweepArgs a) {
+    using G = StarGeo<B, TX, TY, UY, PF>;
+    constexpr int R = G::R, PX = G::PX, NS = G::NS, PAL = G::PLANE_AL, ML = G::ML, WN = G::WN;
+
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    double *ring = reinterpret_cast<double *>(smem_raw);
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * PAL * 8);
+    uint64_t *empty = full + NS;
+
+    const int tile_x = blockIdx.x, tile_y = blockIdx.y;
+    const int chunk = blockIdx.z % a.nchunk;
+    const int64_t prob = blockIdx.z / a.nchunk;
+    const int x0 = a.lo[2] + tile_x * TX, y0 = a.lo[1] + tile_y * TY;
+    const int kb = a.lo[0] + chunk * a.zchunk;
+    const int ke = min(a.hi[0], kb + a.zchunk);
+    if (kb >= ke) return;
+    const int p0 = kb - R, plast = ke - 1 + R;
+    const int64_t zbase = prob * a.nz;
+
+    const int t = threadIdx.x;
+    const int lx = t % G::NTX, ly = t / G::NTX;
+    const int cx = 2 * lx, cy = UY * ly;
+
+    auto issue = [&](int p) {
+        const int slot = (p - p0) % NS;
+        double *dst = ring + slot * PAL;
+        if constexpr (USE_TMA) {
+            if (t == 0) {
+                const int prev = p - NS;
+                if (prev >= p0) mbar_wait(&empty[slot], ((prev - p0) / NS) & 1);
+                mbar_expect_tx(&full[slot], uint32_t(G::PLANE * 8));
+                tma_load_3d(dst, &a.tmap[0], &full[slot], x0 - ML, y0 - R, int(zbase + p));
+            }
+        } else {
+            const int64_t pl = (zbase + p) * a.ny * a.nx;
+            for (int e = t; e < G::PLANE; e += G::THREADS) {
+                const int yy = e / PX, xx = e % PX;
+                const int gx = x0 - ML + xx, gy = y0 - R + yy;
+                const bool ok = gx >= 0 && gx < a.nx && gy >= 0 && gy < a.ny && p >= 0 && p < a.nz;
+                cp_async8(dst + e, a.in[0] + (ok ? pl + int64_t(gy) * a.nx + gx : 0), ok);
+            }
+        }
+    };
+    auto release = [&](int p) {
+        if constexpr (USE_TMA) {
+            __syncwarp();
+            if ((t & 31) == 0)
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[(p - p0) % NS]))
+                             : "memory");
+        }
+    };
+
+    if constexpr (USE_TMA) {
+        if (t == 0) {
+            for (int s = 0; s < NS; s++) {
+                mbar_init(&full[s], 1);
+                mbar_init(&empty[s], G::NWARPS);
+            }
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+        __syncthreads();
+    }
+    for (int p = p0; p < p0 + PF; p++) {
+        if (p <= plast) issue(p);
+        if constexpr (!USE_TMA) cp_async_commit();
+    }
+
+    const int gi = x0 + cx;
+    const bool ok0 = gi >= a.xmin && gi < a.hi[2];
+    const bool ok1 = gi + 1 >= a.xmin && gi + 1 < a.hi[2];
+    const bool vec = ok0 && ok1 && (a.nx % 2 == 0) && ((reinterpret_cast<uintptr_t>(a.out[0]) & 15) == 0);
+    const int nrows = min(UY, a.hi[1] - (y0 + cy));
+
+    double qm[R][UY][2];  // qm[r-1] = centre values of plane k-r
+#pragma unroll
+    for (int r = 0; r < R; r++)
+#pragma unroll
+        for (int py = 0; py < UY; py++) qm[r][py][0] = qm[r][py][1] = 0.0;
+
+    for (int p = p0; p <= plast; p++) {
+        {
+            const int pn = p + PF;
+            if (pn <= plast) issue(pn);
+            if constexpr (!USE_TMA) cp_async_commit();
+        }
+        if constexpr (USE_TMA) {
+            mbar_wait(&full[(p - p0) % NS], ((p - p0) / NS) & 1);
+        } else {
+            cp_async_wait<PF>();
+            __syncthreads();
+        }
+        const int k = p - R;  // plane k is the centre of this iteration
+        if (k >= p0) {
+            const double *cp = ring + ((k - p0) % NS) * PAL;
+            double col[UY + 2 * R][2];  // rows [cy-R, cy+UY+R) of plane k, 2 centre columns
+#pragma unroll
+            for (int r = 0; r < UY + 2 * R; r++) {
+                const double2 v = *reinterpret_cast<const double2 *>(cp + (cy + r) * PX + (cx + ML));
+                col[r][0] = v.x;
+                col[r][1] = v.y;
+            }
+            if (k >= kb) {
+                double acc[UY][2];
+#pragma unroll
+                for (int py = 0; py < UY; py++) acc[py][0] = acc[py][1] = 0.0;
+#pragma unroll
+                for (int r = 1; r <= R; r++) {
+                    const double *up = ring + ((k + r - p0) % NS) * PAL + (cy + R) * PX + (cx + ML);  // plane k+r
+#pragma unroll
+                    for (int py = 0; py < UY; py++) {
+                        const double2 zp = *reinterpret_cast<const double2 *>(up + py * PX);
+                        B::yz(acc[py][0], a, r, (col[py + R + r][0] + col[py + R - r][0]) + (zp.x + qm[r - 1][py][0]));
+                        B::yz(acc[py][1], a, r, (col[py + R + r][1] + col[py + R - r][1]) + (zp.y + qm[r - 1][py][1]));
+                    }
+                }
+#pragma unroll
+                for (int py = 0; py < UY; py++) {
+                    double w[WN];
+                    const double *rp = cp + (cy + py + R) * PX + cx;
+#pragma unroll
+                    for (int c = 0; c < WN / 2; c++) {
+                        const double2 v = *reinterpret_cast<const double2 *>(rp + 2 * c);
+                        w[2 * c] = v.x;
+                        w[2 * c + 1] = v.y;
+                    }
+#pragma unroll
+                    for (int r = 1; r <= R; r++)
+#pragma unroll
+                        for (int px = 0; px < 2; px++) B::x(acc[py][px], a, r, w[ML + px + r] + w[ML + px - r]);
+#pragma unroll
+                    for (int px = 0; px < 2; px++) acc[py][px] = B::finish(acc[py][px], a, w[ML + px]);
+                }
+                release(k);
+                double *o = a.out[0] + ((zbase + k) * a.ny + (y0 + cy)) * a.nx + gi;
+#pragma unroll
+                for (int py = 0; py < UY; py++) {
+                    if (py < nrows) {
+                        if (vec) {
+                            __stcs(reinterpret_cast<double2 *>(o), make_double2(acc[py][0], acc[py][1]));
+                        } else {
+                            if (ok0) __stcs(o, acc[py][0]);
+                            if (ok1) __stcs(o + 1, acc[py][1]);
+                        }
+                    }
+                    o += a.nx;
+                }
+            } else {
+                release(k);  // a plane below the chunk: only feeds the queue
+            }
+            // push plane k's centre values into the register queue
+#pragma unroll
+            for (int r = R - 1; r > 0; r--)
+#pragma unroll
+                for (int py = 0; py < UY; py++) {
+                    qm[r][py][0] = qm[r - 1][py][0];
+                    qm[r][py][1] = qm[r - 1][py][1];
+                }
+#pragma unroll
+            for (int py = 0; py < UY; py++) {
+                qm[0][py][0] = col[py + R][0];
+                qm[0][py][1] = col[py + R][1];
+            }
+        }
+        if constexpr (!USE_TMA) __syncthreads();
     }
 }
 

@@ -1,0 +1,3 @@
+cd $GRAFT_REPO_ROOT
+timeout 900 python tools/perf_sweep.py lap25 --only tma > gpurun_out/perf_sweep.jsonl 2> gpurun_out/perf_sweep.err
+timeout 900 python tools/debug_variants.py 20,34,70 lap25 > gpurun_out/debug_variants.jsonl 2>&1
