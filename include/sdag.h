@@ -84,9 +84,12 @@ typedef struct sdag_plan_opts {
                                   P:1202-1271) -- synchronises the device                  */
     int32_t batch;             /* independent problems per apply (sdag_apply_batched); >= 1 */
     const char *force_variant; /* NULL, or a variant name from sdag_plan_variant_name()    */
+    int32_t fusion;            /* sdag_apply_iterated: 1 = fuse sweeps where a fused kernel
+                                  exists (temporal fusion), 0 = one launch
+                                  per sweep                                               */
 } sdag_plan_opts;
 
-/* Fills `o` with the defaults {order=-1, device=CURRENT, tune=0, batch=1, NULL}. */
+/* Fills `o` with the defaults {order=-1, device=CURRENT, tune=0, batch=1, NULL, fusion=1}. */
 void sdag_plan_opts_init(sdag_plan_opts *o);
 
 typedef struct sdag_plan_info {
@@ -160,6 +163,18 @@ sdag_status sdag_apply_iterated(sdag_plan plan, double *buf0, double *buf1, int3
 sdag_status sdag_apply_host(sdag_plan plan, double *const *host3d, int32_t n3d, const double *const *host1d,
                             int32_t n1d, const double *scalars, int32_t nscalars, sdag_stream stream,
                             int64_t *h2d_bytes, int64_t *d2h_bytes);
+
+/* Pure host logic, no device: the temporal-fusion schedule apply_iterated
+ * uses (NEXT-1; deep tuning's dynamic program, P:1416-1440,
+ * opt(T) = min_x f(x) + opt(T - x)).  f[x], x = 1..maxdeg (f[0] unused), is
+ * the cost of one launch fusing x sweeps; f[x] <= 0 means "no such kernel";
+ * f[1] must be > 0.  Every launch flips a ping-pong pair, so the schedule has
+ * a number of launches with the parity of T (the result lands in buf[T & 1]).
+ * On success seq[0..*n) holds the sweeps per launch in launch order and
+ * *cost their summed f.  Errors: INVALID_ARG for null pointers, maxdeg
+ * outside 1..7, T < 0, f[1] <= 0, or cap < the schedule length. */
+sdag_status sdag_fusion_schedule(const double *f, int32_t maxdeg, int32_t T, int32_t *seq, int32_t cap, int32_t *n,
+                                 double *cost);
 
 /* ------------------------------------------------------------------------
  * a7: z-slab domain decomposition with per-sweep halo exchange

@@ -21,7 +21,7 @@ import os
 from . import _capi
 from ._capi import PlanInfo, PlanOpts, SDAG_DEVICE_CURRENT, SDAG_DEVICE_NONE
 
-__all__ = ["Plan", "Dist", "SdagError", "registry", "spec_text", "slab_partition", "slab_halo", "nccl_unique_id",
+__all__ = ["Plan", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "nccl_unique_id",
            "nccl_comm_create", "nccl_comm_destroy", "launch_count", "fp64_peak", "version", "SPEC_DIR"]
 
 SPEC_DIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "specs")
@@ -67,7 +67,7 @@ def _scal(s):
     return (ctypes.c_double * max(1, len(s)))(*s), len(s)
 
 
-def _opts(order=-1, device=None, tune=False, batch=1, variant=None):
+def _opts(order=-1, device=None, tune=False, batch=1, variant=None, fusion=True):
     o = PlanOpts()
     _capi.lib().sdag_plan_opts_init(ctypes.byref(o))
     o.order = int(order)
@@ -86,6 +86,7 @@ def _opts(order=-1, device=None, tune=False, batch=1, variant=None):
     o.tune = 1 if tune else 0
     o.batch = int(batch)
     o.force_variant = variant.encode() if variant else None
+    o.fusion = 1 if fusion else 0
     return o
 
 
@@ -108,11 +109,11 @@ def spec_text(name: str) -> str:
 class Plan:
     """A planned stencil DAG (a1-a3) bound to grid dims (nz, ny, nx)."""
 
-    def __init__(self, spec: str, dims, order=-1, device=None, tune=False, batch=1, variant=None):
+    def __init__(self, spec: str, dims, order=-1, device=None, tune=False, batch=1, variant=None, fusion=True):
         self._L = _capi.lib()
         self._h = ctypes.c_void_p()
         d = (ctypes.c_int64 * 3)(*[int(x) for x in dims])
-        o = _opts(order, device, tune, batch, variant)
+        o = _opts(order, device, tune, batch, variant, fusion)
         _check(self._L.sdag_plan_create(spec.encode(), d, ctypes.byref(o), ctypes.byref(self._h)))
         self._owned = True
 
@@ -211,6 +212,18 @@ class Plan:
         _check(self._L.sdag_apply_host(self._h, _arr(p3), len(p3), _arr(p1), len(p1), s, ns, _stream_handle(stream),
                                        ctypes.byref(up), ctypes.byref(down)))
         return up.value, down.value
+
+
+def fusion_schedule(f, T: int):
+    """Temporal-fusion schedule (sdag_fusion_schedule): f = {x: cost of an
+    x-sweep launch}; returns (sweeps per launch, total cost)."""
+    maxdeg = max(f)
+    arr = (ctypes.c_double * 8)(*[float(f.get(x, 0.0)) for x in range(8)])
+    cap = max(1, int(T))
+    seq = (ctypes.c_int32 * cap)()
+    n, cost = ctypes.c_int32(), ctypes.c_double()
+    _check(_capi.lib().sdag_fusion_schedule(arr, int(maxdeg), int(T), seq, cap, ctypes.byref(n), ctypes.byref(cost)))
+    return list(seq[:n.value]), cost.value
 
 
 def slab_partition(global_nz: int, rz: int, nranks: int, rank: int) -> dict:

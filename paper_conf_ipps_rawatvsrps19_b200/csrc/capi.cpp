@@ -48,6 +48,7 @@ void sdag_plan_opts_init(sdag_plan_opts *o) {
     o->tune = 0;
     o->batch = 1;
     o->force_variant = nullptr;
+    o->fusion = 1;
 }
 
 sdag_status sdag_plan_create(const char *spec, const int64_t dims[3], const sdag_plan_opts *opts, sdag_plan *out) {
@@ -122,6 +123,24 @@ sdag_status sdag_apply_host(sdag_plan plan, double *const *h3, int32_t n3, const
                             const double *s, int32_t ns, sdag_stream stream, int64_t *h2d, int64_t *d2h) {
     return guard([&] {
         sdag::apply_host(P(plan), h3, n3, h1, n1, s, ns, reinterpret_cast<cudaStream_t>(stream), h2d, d2h);
+    });
+}
+
+sdag_status sdag_fusion_schedule(const double *f, int32_t maxdeg, int32_t T, int32_t *seq, int32_t cap, int32_t *n,
+                                 double *cost) {
+    return guard([&] {
+        if (!f || !seq || !n || !cost) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null pointer");
+        if (maxdeg < 1 || maxdeg > 7 || T < 0) throw sdag::Error(SDAG_ERR_INVALID_ARG, "maxdeg in 1..7, T >= 0");
+        if (!(f[1] > 0.0)) throw sdag::Error(SDAG_ERR_INVALID_ARG, "f[1] must be > 0");
+        const std::vector<int> s = sdag::fusion_schedule(f, maxdeg, T);
+        if (int64_t(s.size()) > cap) throw sdag::Error(SDAG_ERR_INVALID_ARG, "seq capacity too small");
+        double c = 0.0;
+        for (size_t q = 0; q < s.size(); q++) {
+            seq[q] = s[q];
+            c += f[s[q]];
+        }
+        *n = int32_t(s.size());
+        *cost = c;
     });
 }
 

@@ -7,6 +7,7 @@
 #include "bodies.cuh"
 #include "kernels.hpp"
 #include "box27.cuh"
+#include "fuse2.cuh"
 #include "hyp.cuh"
 #include "star.cuh"
 #include "sweep.cuh"
@@ -167,6 +168,38 @@ KernelDesc make_star2_desc(const char *dag, int prio) {
 // code-differencing variants: QMODE 2 = no arithmetic, 3 = no stores (profiling only)
 #define SDAG_STAR_DIFF(v, BODY, DAG, TX, TY, UY, PF, QM, PRIO) \
     v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, QM, 1>(DAG, PRIO))
+
+// two fused sweeps of the 27-point smoother (fuse2.cuh), TMA only
+template <int GX, int GY, int UY, int PF, int MINB = 1>
+KernelDesc make_fuse2_desc(const char *dag, int prio) {
+    using G = dev::Fuse2Geo<GX, GY, UY, PF>;
+    KernelDesc d;
+    d.dag = dag;
+    char buf[96];
+    if (MINB > 1)
+        std::snprintf(buf, sizeof buf, "fuse2_tma_%dx%d_u2x%d_pf%d_mb%d", GX - 2, GY - 2, UY, PF, MINB);
+    else
+        std::snprintf(buf, sizeof buf, "fuse2_tma_%dx%d_u2x%d_pf%d", GX - 2, GY - 2, UY, PF);
+    d.variant = buf;
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_box27x2<GX, GY, UY, PF, MINB>);
+    d.threads = G::THREADS;
+    d.smem = G::SMEM;
+    d.tx = GX - 2;
+    d.ty = GY - 2;
+    d.ux = 2;
+    d.uy = UY;
+    d.pf = PF;
+    d.tma = true;
+    d.nin = 1;
+    d.nout = 1;
+    d.rz = 1;
+    d.ry = 2;  // TMA box (GY+2) = ty + 2*ry
+    d.rx = 3;  // TMA box (GX+4) = tx + 2*rx, origin tile-3 (even)
+    d.rzr = 2;
+    d.prio = prio;
+    d.tsteps = 2;
+    return d;
+}
 
 // phase-unrolled queue (QMODE 1), TMA only
 #define SDAG_STARQ(v, BODY, DAG, TX, TY, UY, PF, PRIO) \

@@ -18,6 +18,7 @@ struct KernelDesc {
     int nin = 0, nout = 0, nio = 0, n1d = 0;
     int rz = 0, ry = 0, rx = 0, rzr = 0;  // body radius and shared-memory ring z-window
     int prio = 0;                         // heuristic preference (lower first)
+    int tsteps = 1;                       // sweeps fused per launch (temporal fusion, NEXT-1)
 };
 
 // all kernels, in heuristic preference order per DAG

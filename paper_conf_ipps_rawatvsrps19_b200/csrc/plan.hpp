@@ -40,6 +40,9 @@ struct Plan {
     // ABI mapping (per 3D formal kind_index): staged-input slot / output slot / inout slot
     std::vector<int> in_slot, out_slot, io_slot;
     std::vector<const KernelDesc *> cands;  // candidate kernels (TMA first)
+    std::vector<const KernelDesc *> fused;  // multi-sweep kernels for apply_iterated (tsteps > 1)
+    double fcost[8] = {0};                  // f(x): relative cost of an x-sweep launch (deep tuning)
+    bool fusion = true;                     // use fused kernels in apply_iterated
     int chosen = -1;                        // index into cands
     std::string describe_text;
 
@@ -69,6 +72,7 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *arrays3d, const do
                  const int64_t *dims_override = nullptr);
 void apply(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns, int batch,
            cudaStream_t stream);
+std::vector<int> fusion_schedule(const double *f, int maxdeg, int T);
 void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int ns, cudaStream_t stream);
 void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int n1, const double *s, int ns,
                 cudaStream_t stream, int64_t *h2d, int64_t *d2h);

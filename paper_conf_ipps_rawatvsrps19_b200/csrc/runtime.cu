@@ -5,6 +5,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <array>
 #include <atomic>
 #include <cmath>
 #include <cstring>
@@ -308,6 +309,37 @@ void apply(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, 
     plan_launch(p, k, a3, a1, s, batch, 0, p->dims[0], stream);
 }
 
+// Fusion schedule for T sweeps (deep tuning): degrees x with
+// costs f(x); opt(T) = min_x f(x) + opt(T - x), constrained so
+// that the number of launches has the parity of T (each launch flips the
+// ping-pong buffer; the result must land in buf[T&1]).
+std::vector<int> fusion_schedule(const double *f, int maxdeg, int T) {
+    const double INF = 1e300;
+    std::vector<std::array<double, 2>> best(T + 1, {INF, INF});
+    std::vector<std::array<int, 2>> pick(T + 1, {0, 0});
+    best[0][0] = 0.0;
+    for (int t = 1; t <= T; t++)
+        for (int q = 0; q < 2; q++)
+            for (int d = 1; d <= std::min(maxdeg, t); d++) {
+                if (f[d] <= 0.0) continue;
+                const double c = f[d] + best[t - d][1 - q];
+                if (c < best[t][q]) {
+                    best[t][q] = c;
+                    pick[t][q] = d;
+                }
+            }
+    std::vector<int> seq;
+    int t = T, q = T & 1;
+    while (t > 0) {
+        const int d = pick[t][q];
+        if (d <= 0) throw Error(SDAG_ERR_INVALID_ARG, "no fusion schedule");
+        seq.push_back(d);
+        t -= d;
+        q ^= 1;
+    }
+    return seq;
+}
+
 void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int ns, cudaStream_t stream) {
     if (p->n3() != 2 || p->an.n_in != 1 || p->an.n_out != 1 || p->n1() != 0)
         throw Error(SDAG_ERR_INVALID_ARG, "apply_iterated needs a 1-input 1-output plan without 1D arrays");
@@ -316,11 +348,34 @@ void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int
     int fin = -1, fout = -1;
     for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
     double *bufs[2] = {b0, b1};
-    for (int t = 0; t < T; t++) {
+    // fused kernels need the TMA path and the plan's dims
+    int maxdeg = 1;
+    const KernelDesc *fk[8] = {nullptr};
+    if (p->fusion && !p->fused.empty() && tma_ok(p, bufs, p->dims[2]) &&
+        (reinterpret_cast<uintptr_t>(b0) % 16) == 0 && (reinterpret_cast<uintptr_t>(b1) % 16) == 0) {
+        for (const KernelDesc *f : p->fused)
+            if (!fk[f->tsteps]) {
+                fk[f->tsteps] = f;
+                maxdeg = std::max(maxdeg, f->tsteps);
+            }
+    }
+    double f[8];
+    for (int d = 0; d < 8; d++) f[d] = (d == 1 || (d > 1 && d <= maxdeg && fk[d])) ? p->fcost[d] : 0.0;
+    const std::vector<int> seq = fusion_schedule(f, maxdeg, T);
+    int cur = 0;
+    for (int d : seq) {
         double *a3[2];
-        a3[fin] = bufs[t & 1];
-        a3[fout] = bufs[(t + 1) & 1];
-        apply(p, a3, 2, nullptr, 0, s, ns, 1, stream);
+        a3[fin] = bufs[cur];
+        a3[fout] = bufs[1 - cur];
+        if (d == 1) {
+            apply(p, a3, 2, nullptr, 0, s, ns, 1, stream);
+        } else {
+            if (ns != p->ns()) throw Error(SDAG_ERR_INVALID_ARG, "scalar count");
+            validate_arrays(p, a3, 2, nullptr, 0, ns, p->dims[0] * p->dims[1] * p->dims[2]);
+            DeviceGuard g(p);
+            plan_launch(p, *fk[d], a3, nullptr, s, 1, 0, p->dims[0], stream);
+        }
+        cur = 1 - cur;
     }
 }
 
@@ -427,6 +482,7 @@ Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_pla
     }
     p->batch_hint = std::max(1, o.batch);
     p->tune = o.tune;
+    p->fusion = o.fusion != 0;
     if (o.force_variant) p->force_variant = o.force_variant;
 
     // device
@@ -476,8 +532,19 @@ Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_pla
         // code-differencing variants compute something else on purpose:
         // only reachable through force_variant
         if (k.prio >= 1000 && k.variant != p->force_variant) continue;
+        if (k.tsteps > 1) {  // temporal fusion kernels serve apply_iterated only
+            p->fused.push_back(&k);
+            continue;
+        }
         p->cands.push_back(&k);
     }
+    std::stable_sort(p->fused.begin(), p->fused.end(),
+                     [](const KernelDesc *a, const KernelDesc *b) { return a->prio < b->prio; });
+    // f(x) of the deep-tuning DP: default estimate for a
+    // bandwidth-bound stencil -- an x-sweep launch moves the data of one sweep
+    // plus overlapped-tiling overhead; replaced by measured times when tune=1
+    p->fcost[1] = 1.0;
+    for (const KernelDesc *f : p->fused) p->fcost[f->tsteps] = 1.0 + 0.15 * (f->tsteps - 1);
     std::stable_sort(p->cands.begin(), p->cands.end(),
                      [](const KernelDesc *a, const KernelDesc *b) { return a->prio < b->prio; });
     if (p->cands.empty()) throw Error(SDAG_ERR_UNSUPPORTED, "no kernel variant fits this plan");
@@ -486,6 +553,12 @@ Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_pla
         p->chosen = -1;
         for (size_t q = 0; q < p->cands.size(); q++)
             if (p->cands[q]->variant == p->force_variant) p->chosen = int(q);
+        for (const KernelDesc *f : p->fused)  // forcing a fused kernel pins apply_iterated's fusion
+            if (f->variant == p->force_variant) {
+                p->fused = {f};
+                p->chosen = 0;
+                break;
+            }
         if (p->chosen < 0) throw Error(SDAG_ERR_INVALID_ARG, "unknown variant '" + p->force_variant + "'");
     } else if (p->tune && !p->host_only) {
         time_candidates(p.get());
@@ -495,6 +568,13 @@ Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_pla
     d << "\n  variant " << k.variant << " (" << k.threads << " threads, " << k.smem << " B smem, ring "
       << (2 * k.rzr + 1 + k.pf) << " planes)" << (p->tune ? "  [tuned]" : "  [heuristic]") << "\n  candidates:";
     for (auto *c : p->cands) d << " " << c->variant;
+    if (!p->fused.empty()) {
+        d << "\n  temporal fusion (apply_iterated):";
+        for (auto *c : p->fused) d << " " << c->variant << " [" << c->tsteps << " sweeps]";
+        d << "\n  f(x) per launch relative to one sweep" << (p->tune ? " (measured)" : " (estimate)") << ":";
+        for (int x = 1; x < 8; x++)
+            if (p->fcost[x] > 0.0) d << " f(" << x << ")=" << p->fcost[x];
+    }
     p->describe_text = d.str();
     return p.release();
 }
@@ -548,9 +628,32 @@ static void time_candidates(Plan *p) {
                 bestq = int(q);
             }
         }
+        p->chosen = bestq;
+        // deep tuning: measure f(x) of every fused x-sweep kernel
+        // relative to the chosen single sweep, fastest fused kernel per x first
+        if (!p->fused.empty() && p->dims[2] % 2 == 0 && best < 1e29f) {
+            std::vector<std::pair<float, const KernelDesc *>> tf;
+            for (const KernelDesc *f : p->fused) {
+                plan_launch(p, *f, b3.data(), b1.data(), s.data(), 1, 0, p->dims[0], 0);
+                check_cuda(cudaEventRecord(e0, 0), "event");
+                for (int r = 0; r < 3; r++) plan_launch(p, *f, b3.data(), b1.data(), s.data(), 1, 0, p->dims[0], 0);
+                check_cuda(cudaEventRecord(e1, 0), "event");
+                check_cuda(cudaEventSynchronize(e1), "event sync");
+                float ms = 0;
+                check_cuda(cudaEventElapsedTime(&ms, e0, e1), "event time");
+                tf.push_back({ms, f});
+            }
+            std::stable_sort(tf.begin(), tf.end(), [](auto &a, auto &b) { return a.first < b.first; });
+            const double single = best / double(p->batch_hint);
+            for (int d = 2; d < 8; d++) p->fcost[d] = 0.0;
+            p->fused.clear();
+            for (auto &[ms, f] : tf) {
+                if (p->fcost[f->tsteps] == 0.0) p->fcost[f->tsteps] = ms / single;
+                p->fused.push_back(f);
+            }
+        }
         cudaEventDestroy(e0);
         cudaEventDestroy(e1);
-        p->chosen = bestq;
     } catch (...) {
         cleanup();
         throw;

@@ -347,3 +347,55 @@ def test_full_size_smooth27_iterated_sampled():
         ab = oracle.smooth27_iter_points(np.abs(box), np.abs(w), nu, T, lp, absmode=True)
         g = res[int(p[0]), int(p[1]), int(p[2])].item()
         assert scaled_err([g], o, ab) <= T * TOL, (p, g, o)
+
+
+FUSED = ["fuse2_tma_62x14_u2x2_pf2", "fuse2_tma_30x14_u2x2_pf2_mb3", "fuse2_tma_126x14_u2x4_pf2", "fuse2_tma_62x30_u2x2_pf2",
+         "fuse2_tma_126x14_u2x2_pf2"]
+
+
+@pytest.mark.parametrize("variant", FUSED)
+@pytest.mark.parametrize("dims", [(26, 30, 40), (33, 20, 132), (9, 70, 260)], ids=lambda d: "x".join(map(str, d)))
+def test_temporal_fusion_matches_oracle_and_unfused(variant, dims):
+    """NEXT-1: two sweeps per launch (overlapped tiling in x/y, retimed z);
+    the DP schedule mixes 2-sweep and 1-sweep launches to keep the ping-pong
+    parity.  Same result as T single sweeps (and the oracle) for odd and even T."""
+    ins, sc = synth.smooth27_inputs(dims, cfg="fuse")
+    A = ins["A"]
+    w = [sc[k] for k in ("w0", "w1", "w2", "w3")]
+    s = [*w, sc["nu"]]
+    fused = sdag.Plan(sdag.spec_text("smooth27"), dims, variant=variant)
+    plain = sdag.Plan(sdag.spec_text("smooth27"), dims, fusion=False)
+    for T in (1, 2, 3, 5, 12):
+        outs = []
+        for plan in (fused, plain):
+            b0 = torch.from_numpy(A).cuda()
+            b1 = b0.clone()
+            n0 = sdag.launch_count()
+            plan.apply_iterated(b0, b1, T, scalars=s)
+            torch.cuda.synchronize()
+            outs.append(((b0 if T % 2 == 0 else b1).cpu().numpy(), sdag.launch_count() - n0))
+        (gf, nf), (gp, np_) = outs
+        # launches flip the ping-pong pair once each, so #launches == T (mod 2)
+        assert np_ == T and nf == {1: 1, 2: 2, 3: 3, 5: 3, 12: 6}[T]
+        O = oracle.smooth27_iter(A, w, sc["nu"], T)
+        Aabs = oracle.smooth27_iter(np.abs(A), np.abs(w), sc["nu"], T, absmode=True)
+        assert scaled_err(gf, O, Aabs) <= T * TOL
+        assert scaled_err(gp, O, Aabs) <= T * TOL
+        assert np.array_equal(gf[ring_mask(dims, 1)], A[ring_mask(dims, 1)])
+
+
+def test_temporal_fusion_exact_closed_form():
+    """V8 through the fused kernels: integer weights, quadratic input, bit-exact."""
+    dims, T = (16, 18, 20), 4
+    k, j, i = np.meshgrid(*[np.arange(n, dtype=np.float64) - n // 2 for n in dims], indexing="ij")
+    p = 3 * i * i - 2 * j * j + 5 * k * k + i * j - 3 * j * k + 2 * i + 11
+    plan = sdag.Plan(sdag.spec_text("smooth27"), dims)
+    assert "temporal fusion" in plan.describe()
+    b0 = torch.from_numpy(p.copy()).cuda()
+    b1 = b0.clone()
+    n0 = sdag.launch_count()
+    plan.apply_iterated(b0, b1, T, scalars=[-128.0, 14.0, 3.0, 1.0, 1.0 / 32.0])
+    torch.cuda.synchronize()
+    assert sdag.launch_count() - n0 == 2  # two fused launches
+    G = b0.cpu().numpy()
+    assert np.array_equal(G, oracle.smooth27_iter(p, [-128.0, 14.0, 3.0, 1.0], 1 / 32, T))
