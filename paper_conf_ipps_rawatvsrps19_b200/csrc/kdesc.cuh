@@ -44,16 +44,19 @@ KernelDesc make_desc(const char *dag, int prio) {
 }
 
 // star-stencil kernel (star.cuh): 2-wide x patch, UY-tall y patch, register z-queue
-template <class B, int TX, int TY, int UY, int PF, bool TMA, int QMODE = 0, int MINB = 1>
+template <class B, int TX, int TY, int UY, int PF, bool TMA, int QMODE = 0, int MINB = 1, int UNR = 1>
 KernelDesc make_star_desc(const char *dag, int prio) {
     using G = dev::StarGeo<B, TX, TY, UY, PF>;
     KernelDesc d;
     d.dag = dag;
     char buf[96];
-    std::snprintf(buf, sizeof buf, "star%s_%s_%dx%d_u2x%d_pf%d%s", QMODE == 1 ? "q" : (QMODE == 2 ? "DIFFmem" : (QMODE == 3 ? "DIFFnost" : "")), TMA ? "tma" : "lsu", TX, TY, UY, PF,
-                  MINB > 1 ? (MINB == 2 ? "_mb2" : "_mb3") : "");
+    char unr[16] = "";
+    if (UNR > 1) std::snprintf(unr, sizeof unr, "_z%d", UNR);
+    std::snprintf(buf, sizeof buf, "star%s_%s_%dx%d_u2x%d_pf%d%s%s",
+                  QMODE == 1 ? "q" : (QMODE == 2 ? "DIFFmem" : (QMODE == 3 ? "DIFFnost" : (QMODE == 4 ? "L" : (QMODE == 5 ? "S" : (QMODE == 6 ? "R" : ""))))), TMA ? "tma" : "lsu", TX,
+                  TY, UY, PF, MINB > 1 ? (MINB == 2 ? "_mb2" : "_mb3") : "", unr);
     d.variant = buf;
-    d.fn = reinterpret_cast<const void *>(&dev::sdag_star<B, TX, TY, UY, PF, TMA, QMODE, MINB>);
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_star<B, TX, TY, UY, PF, TMA, QMODE, MINB, UNR>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = TX;
@@ -166,6 +169,32 @@ KernelDesc make_star2_desc(const char *dag, int prio) {
     } while (0)
 
 // code-differencing variants: QMODE 2 = no arithmetic, 3 = no stores (profiling only)
+// plane-loop unroll UNR (queue shifted once per UNR planes), TMA + LSU twin
+#define SDAG_STAR_UNR(v, BODY, DAG, TX, TY, UY, PF, MB, UNR, PRIO)                                \
+    do {                                                                                          \
+        v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, 0, MB, UNR>(DAG, PRIO));       \
+        v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, false, 0, MB, UNR>(DAG, PRIO + 100)); \
+    } while (0)
+
+// late-head variant (QMODE 4, TMA only)
+#define SDAG_STAR_LATE(v, BODY, DAG, TX, TY, UY, PF, MB, UNR, PRIO) \
+    v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, 4, MB, UNR>(DAG, PRIO))
+
+// split-accumulator variant (QMODE 5) + LSU twin
+#define SDAG_STAR_SPLIT(v, BODY, DAG, TX, TY, UY, PF, MB, UNR, PRIO)                                \
+    do {                                                                                            \
+        v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, 5, MB, UNR>(DAG, PRIO));         \
+        v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, false, 5, MB, UNR>(DAG, PRIO + 100));  \
+    } while (0)
+
+// rotating-queue variant (QMODE 6, plane loop unrolled by 2R+1) + LSU twin
+#define SDAG_STAR_ROT(v, BODY, DAG, TX, TY, UY, PF, MB, PRIO)                                              \
+    do {                                                                                                   \
+        v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, 6, MB, 2 * dev::BODY::R + 1>(DAG, PRIO)); \
+        v.push_back(                                                                                       \
+            make_star_desc<dev::BODY, TX, TY, UY, PF, false, 6, MB, 2 * dev::BODY::R + 1>(DAG, PRIO + 100));  \
+    } while (0)
+
 #define SDAG_STAR_DIFF(v, BODY, DAG, TX, TY, UY, PF, QM, PRIO) \
     v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, QM, 1>(DAG, PRIO))
 

@@ -19,9 +19,19 @@
 // warp) instead of a CTA-wide barrier per plane, so warps do not wait for one
 // another; only the TMA-issuing thread waits for a slot to drain.
 //
-// QMODE 0: the queue is shifted with register moves after every plane;
+// QMODE 0: the queue is shifted with register moves; with UNR > 1 the plane
+//   loop is unrolled UNR times over a queue of NQ + UNR - 1 slots, so the
+//   (NQ - 1)-slot shift happens once per UNR planes (UNR x the code, 1/UNR of
+//   the moves);
 // QMODE 1: the plane loop is dispatched to NQ phase copies so the queue
-// rotates by compile-time indexing (no moves, NQ x the code).
+// rotates by compile-time indexing (no moves, NQ x the code);
+// QMODE 4 ("late head", TMA): as QMODE 0, but plane p's barrier is only probed
+//   (mbarrier.test_wait) at the start of its step; all taps of output k = p-R
+//   except the z-tap at p are computed first, and the warp spins only if the
+//   plane has still not landed -- the barrier latency leaves the critical path;
+// QMODE 5: as QMODE 0 with the x taps in a separate accumulator chain;
+// QMODE 6: the plane loop unrolled by the queue depth NQ (UNR == NQ): plane
+//   p lives in slot (p - p0) mod NQ for its whole life, no moves, no dispatch.
 //
 // Arithmetic is re-associated relative to the spec (y/z taps first, then x,
 // then the centre, each group as fma(c_r, sum, acc)); parity is by the scaled
@@ -92,7 +102,7 @@ struct StarGeo {
     static_assert(PX <= 256 && PY <= 256, "TMA box");
 };
 
-template <class B, int TX, int TY, int UY, int PF, bool USE_TMA, int QMODE = 0, int MINB = 1>
+template <class B, int TX, int TY, int UY, int PF, bool USE_TMA, int QMODE = 0, int MINB = 1, int UNR = 1>
 __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
     sdag_star(const __grid_constant__ SweepArgs a) {
     using G = StarGeo<B, TX, TY, UY, PF>;
@@ -119,13 +129,13 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
     const int cy = UY * ly;  // patch y offset inside the tile
 
     auto issue = [&](int p) {
-        const int slot = (p - p0) % NS;
+        const int slot = unsigned(p - p0) % NS;
         double *dst = ring + slot * PAL;
         if constexpr (USE_TMA) {
             if (t == 0) {
                 // the previous occupant, plane p-NS, must have been released by every warp
                 const int prev = p - NS;
-                if (prev >= p0) mbar_wait(&empty[slot], ((prev - p0) / NS) & 1);
+                if (prev >= p0) mbar_wait(&empty[slot], (unsigned(prev - p0) / NS) & 1);
                 mbar_expect_tx(&full[slot], uint32_t(G::PLANE * 8));
                 tma_load_3d(dst, &a.tmap[0], &full[slot], x0 - ML, y0 - R, int(zbase + p));
             }
@@ -143,7 +153,7 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
         if constexpr (USE_TMA) {
             __syncwarp();
             if ((t & 31) == 0)
-                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[(p - p0) % NS]))
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[unsigned(p - p0) % NS]))
                              : "memory");
         }
     };
@@ -170,7 +180,12 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
     const bool vec = ok0 && ok1 && (a.nx % 2 == 0) && ((reinterpret_cast<uintptr_t>(a.out[0]) & 15) == 0);
     const int nrows = min(UY, a.hi[1] - (y0 + cy));
 
-    double q[NQ][UY][2];  // register z-queue (see QMODE)
+    constexpr bool ROT = QMODE == 1 || QMODE == 6;  // queue rotates by indexing, no moves
+    static_assert(QMODE != 6 || UNR == NQ, "QMODE 6 unrolls the plane loop by the queue depth");
+    constexpr int NQS = ROT ? NQ : NQ + UNR - 1;
+    double q[NQS][UY][2];  // register z-queue (see QMODE)
+    // queue slot of plane k + d (k = p - R) when plane p sits in slot PH
+    auto qs = [](int ph, int d) { return ROT ? (ph + NQ - R + d) % NQ : ph - R + d; };
 
     auto step = [&](auto phase, int p) {
         constexpr int PH = decltype(phase)::value;  // slot of plane p in q
@@ -179,14 +194,104 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
             if (pn <= plast) issue(pn);
             if constexpr (!USE_TMA) cp_async_commit();
         }
+        if constexpr (QMODE == 4) {
+            // late head (TMA only): the centre plane k = p - R has been resident
+            // for R planes, so everything but the z-tap at k+R = p is computed
+            // while plane p's barrier is probed; the warp spins (if at all)
+            // only after that work, then folds in plane p's centre values.
+            const int slot = unsigned(p - p0) % NS;
+            const uint32_t par = (unsigned(p - p0) / NS) & 1;
+            const bool ready = mbar_test(&full[slot], par);
+            const int k = p - R;
+            const double *hp = ring + slot * PAL + (cy + R) * PX + (cx + ML);
+            if (k >= kb) {
+                const double *cp = ring + (unsigned(k - p0) % NS) * PAL;
+                double acc[UY][2], last[UY][2];
+                double col[UY + 2 * R][2];
+#pragma unroll
+                for (int r = 0; r < UY + 2 * R; r++) {
+                    const double2 v = *reinterpret_cast<const double2 *>(cp + (cy + r) * PX + (cx + ML));
+                    col[r][0] = v.x;
+                    col[r][1] = v.y;
+                }
+#pragma unroll
+                for (int py = 0; py < UY; py++)
+#pragma unroll
+                    for (int px = 0; px < 2; px++) {
+                        acc[py][px] = 0.0;
+                        last[py][px] = (col[py + 2 * R][px] + col[py][px]) + q[qs(PH, -R)][py][px];
+                    }
+#pragma unroll
+                for (int r = 1; r < R; r++)
+#pragma unroll
+                    for (int py = 0; py < UY; py++)
+#pragma unroll
+                        for (int px = 0; px < 2; px++) {
+                            const double zp = q[qs(PH, r)][py][px];
+                            const double zm = q[qs(PH, -r)][py][px];
+                            B::yz(acc[py][px], a, r, (col[py + R + r][px] + col[py + R - r][px]) + (zp + zm));
+                        }
+#pragma unroll
+                for (int py = 0; py < UY; py++) {
+                    double w[WN];
+                    const double *rp = cp + (cy + py + R) * PX + cx;
+#pragma unroll
+                    for (int c = 0; c < WN / 2; c++) {
+                        const double2 v = *reinterpret_cast<const double2 *>(rp + 2 * c);
+                        w[2 * c] = v.x;
+                        w[2 * c + 1] = v.y;
+                    }
+#pragma unroll
+                    for (int r = 1; r <= R; r++)
+#pragma unroll
+                        for (int px = 0; px < 2; px++) B::x(acc[py][px], a, r, w[ML + px + r] + w[ML + px - r]);
+                }
+                release(k);  // last use of plane k (as centre)
+                if (!ready) mbar_wait(&full[slot], par);
+#pragma unroll
+                for (int py = 0; py < UY; py++) {
+                    const double2 v = *reinterpret_cast<const double2 *>(hp + py * PX);
+                    q[PH][py][0] = v.x;
+                    q[PH][py][1] = v.y;
+#pragma unroll
+                    for (int px = 0; px < 2; px++) {
+                        B::yz(acc[py][px], a, R, last[py][px] + q[PH][py][px]);
+                        acc[py][px] = B::finish(acc[py][px], a, col[py + R][px]);
+                    }
+                }
+                double *o = a.out[0] + ((zbase + k) * a.ny + (y0 + cy)) * a.nx + gi;
+#pragma unroll
+                for (int py = 0; py < UY; py++) {
+                    if (py < nrows) {
+                        if (vec) {
+                            __stcs(reinterpret_cast<double2 *>(o), make_double2(acc[py][0], acc[py][1]));
+                        } else {
+                            if (ok0) __stcs(o, acc[py][0]);
+                            if (ok1) __stcs(o + 1, acc[py][1]);
+                        }
+                    }
+                    o += a.nx;
+                }
+            } else {
+                if (!ready) mbar_wait(&full[slot], par);
+#pragma unroll
+                for (int py = 0; py < UY; py++) {
+                    const double2 v = *reinterpret_cast<const double2 *>(hp + py * PX);
+                    q[PH][py][0] = v.x;
+                    q[PH][py][1] = v.y;
+                }
+                if (p < kb) release(p);  // a head-only plane (never a centre) is done
+            }
+            return;
+        }
         if constexpr (USE_TMA) {
-            mbar_wait(&full[(p - p0) % NS], ((p - p0) / NS) & 1);
+            mbar_wait(&full[unsigned(p - p0) % NS], (unsigned(p - p0) / NS) & 1);
         } else {
             cp_async_wait<PF>();
             __syncthreads();
         }
         {  // queue head: plane p's centre values
-            const double *hp = ring + ((p - p0) % NS) * PAL + (cy + R) * PX + (cx + ML);
+            const double *hp = ring + (unsigned(p - p0) % NS) * PAL + (cy + R) * PX + (cx + ML);
 #pragma unroll
             for (int py = 0; py < UY; py++) {
                 const double2 v = *reinterpret_cast<const double2 *>(hp + py * PX);
@@ -196,11 +301,11 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
         }
         const int k = p - R;
         if (k >= kb) {
-            const double *cp = ring + ((k - p0) % NS) * PAL;  // centre plane k with its xy halo
+            const double *cp = ring + (unsigned(k - p0) % NS) * PAL;  // centre plane k with its xy halo
             double acc[UY][2];
 #pragma unroll
             for (int py = 0; py < UY; py++) acc[py][0] = acc[py][1] = 0.0;
-            if constexpr (QMODE >= 2 && QMODE != 3) {
+            if constexpr (QMODE == 2) {
                 // code differencing: memory pipeline only, no stencil arithmetic
 #pragma unroll
                 for (int py = 0; py < UY; py++) acc[py][0] = q[PH][py][0], acc[py][1] = q[PH][py][1];
@@ -222,8 +327,8 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
 #pragma unroll
                         for (int px = 0; px < 2; px++) {
                             // plane k+d (k = p-R) lives in slot (PH - R + d) mod NQ
-                            const double zp = q[(PH + NQ - R + r) % NQ][py][px];
-                            const double zm = q[(PH + NQ - R - r) % NQ][py][px];
+                            const double zp = q[qs(PH, r)][py][px];
+                            const double zm = q[qs(PH, -r)][py][px];
                             B::yz(acc[py][px], a, r, (col[py + R + r][px] + col[py + R - r][px]) + (zp + zm));
                         }
             }
@@ -239,12 +344,24 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
                     w[2 * c] = v.x;
                     w[2 * c + 1] = v.y;
                 }
+                if constexpr (QMODE == 5) {
+                    // split accumulators: x taps in their own chain, joined
+                    // before the centre term (dependency depth 2R+2, not 2R+1+...)
+                    double ax[2] = {0.0, 0.0};
 #pragma unroll
-                for (int r = 1; r <= R; r++)
+                    for (int r = 1; r <= R; r++)
 #pragma unroll
-                    for (int px = 0; px < 2; px++) B::x(acc[py][px], a, r, w[ML + px + r] + w[ML + px - r]);
+                        for (int px = 0; px < 2; px++) B::x(ax[px], a, r, w[ML + px + r] + w[ML + px - r]);
 #pragma unroll
-                for (int px = 0; px < 2; px++) acc[py][px] = B::finish(acc[py][px], a, w[ML + px]);
+                    for (int px = 0; px < 2; px++) acc[py][px] = B::finish(acc[py][px] + ax[px], a, w[ML + px]);
+                } else {
+#pragma unroll
+                    for (int r = 1; r <= R; r++)
+#pragma unroll
+                        for (int px = 0; px < 2; px++) B::x(acc[py][px], a, r, w[ML + px + r] + w[ML + px - r]);
+#pragma unroll
+                    for (int px = 0; px < 2; px++) acc[py][px] = B::finish(acc[py][px], a, w[ML + px]);
+                }
             }
             }
             release(k);  // last use of plane k (as centre)
@@ -269,20 +386,28 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
         if constexpr (!USE_TMA) __syncthreads();  // the LSU ring has no empty barriers
     };
 
-    if constexpr (QMODE == 0) {
-        for (int p = p0; p <= plast; p++) {
-            step(std::integral_constant<int, NQ - 1>{}, p);
+    if constexpr (QMODE == 6) {
+        for (int p = p0; p <= plast; p += NQ)
+            static_for<NQ>([&](auto I) {
+                if (p + decltype(I)::value <= plast) step(I, p + decltype(I)::value);
+            });
+    } else if constexpr (QMODE != 1) {
+        for (int p = p0; p <= plast; p += UNR) {
+            static_for<UNR>([&](auto I) {
+                if (UNR == 1 || p + decltype(I)::value <= plast)
+                    step(std::integral_constant<int, NQ - 1 + decltype(I)::value>{}, p + decltype(I)::value);
+            });
 #pragma unroll
             for (int d = 0; d < NQ - 1; d++)
 #pragma unroll
                 for (int py = 0; py < UY; py++) {
-                    q[d][py][0] = q[d + 1][py][0];
-                    q[d][py][1] = q[d + 1][py][1];
+                    q[d][py][0] = q[d + UNR][py][0];
+                    q[d][py][1] = q[d + UNR][py][1];
                 }
         }
     } else {
         for (int p = p0; p <= plast; p++) {
-            const int ph = (p - p0) % NQ;
+            const int ph = unsigned(p - p0) % NQ;
             static_for<NQ>([&](auto I) {
                 if (ph == decltype(I)::value) step(I, p);
             });
@@ -322,12 +447,12 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
     const int cx = 2 * lx, cy = UY * ly;
 
     auto issue = [&](int p) {
-        const int slot = (p - p0) % NS;
+        const int slot = unsigned(p - p0) % NS;
         double *dst = ring + slot * PAL;
         if constexpr (USE_TMA) {
             if (t == 0) {
                 const int prev = p - NS;
-                if (prev >= p0) mbar_wait(&empty[slot], ((prev - p0) / NS) & 1);
+                if (prev >= p0) mbar_wait(&empty[slot], (unsigned(prev - p0) / NS) & 1);
                 mbar_expect_tx(&full[slot], uint32_t(G::PLANE * 8));
                 tma_load_3d(dst, &a.tmap[0], &full[slot], x0 - ML, y0 - R, int(zbase + p));
             }
@@ -345,7 +470,7 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
         if constexpr (USE_TMA) {
             __syncwarp();
             if ((t & 31) == 0)
-                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[(p - p0) % NS]))
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[unsigned(p - p0) % NS]))
                              : "memory");
         }
     };
@@ -384,14 +509,14 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
             if constexpr (!USE_TMA) cp_async_commit();
         }
         if constexpr (USE_TMA) {
-            mbar_wait(&full[(p - p0) % NS], ((p - p0) / NS) & 1);
+            mbar_wait(&full[unsigned(p - p0) % NS], (unsigned(p - p0) / NS) & 1);
         } else {
             cp_async_wait<PF>();
             __syncthreads();
         }
         const int k = p - R;  // plane k is the centre of this iteration
         if (k >= p0) {
-            const double *cp = ring + ((k - p0) % NS) * PAL;
+            const double *cp = ring + (unsigned(k - p0) % NS) * PAL;
             double col[UY + 2 * R][2];  // rows [cy-R, cy+UY+R) of plane k, 2 centre columns
 #pragma unroll
             for (int r = 0; r < UY + 2 * R; r++) {
