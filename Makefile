@@ -10,7 +10,7 @@ LIB     := $(LIBDIR)/libsdag.so
 ARCH    := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -Wall -Iinclude -I$(SRC) -I$(BUILD) \
            --expt-relaxed-constexpr
-CU_SRCS := k_jacobi7 k_lap25 k_smooth27 k_hypterm k_rhs4 k_toys runtime
+CU_SRCS := k_jacobi7 k_lap25 k_smooth27 k_hypterm k_rhs4 k_toys runtime jit
 CC_SRCS := spec analysis registry dist capi
 OBJS    := $(addprefix $(BUILD)/,$(addsuffix .o,$(CU_SRCS) $(CC_SRCS)))
 HDRS    := $(wildcard $(SRC)/*.hpp $(SRC)/*.cuh) include/sdag.h
@@ -26,6 +26,12 @@ $(BUILD)/%.o: $(SRC)/%.cu $(HDRS)
 	$(NVCC) $(NVFLAGS) -c $< -o $@
 
 $(BUILD)/registry.o: $(BUILD)/specs_embed.inc
+
+$(BUILD)/jit_embed.inc: $(SRC)/sweep.cuh tools/embed_text.py
+	@mkdir -p $(BUILD)
+	$(PY) tools/embed_text.py $@ kSweepSrc $(SRC)/sweep.cuh
+
+$(BUILD)/jit.o: $(BUILD)/jit_embed.inc
 
 $(BUILD)/%.o: $(SRC)/%.cpp $(HDRS)
 	@mkdir -p $(BUILD)

@@ -1,0 +1,380 @@
+// jit.cu -- NEXT-4: arbitrary single-stage stencil DAGs on the
+// GPU by run-time code generation.
+//
+// The paper's framework is a code generator: a DSL spec becomes CUDA source
+// (Listing 2).  For DAGs without a hand-written sm_100a body in the
+// registry, this file does the same at plan time, B200-style:
+//   1. the resolved IR (ir.hpp) is printed as a point body -- one C++
+//      expression per statement, fully parenthesised in program order, literals
+//      as exact hexadecimal doubles, loads as ring taps g.at(slot,dz,dy,dx),
+//      1D arrays as g.s1, scalars as g.s, inout reads-before-write as g.io,
+//      reads of an array after its write as the value just computed (the
+//      semantics of reading R3 / SURVEY 8(c) c1);
+//   2. NVRTC compiles that body into the same z-streaming TMA/LSU skeleton
+//      (sweep.cuh, embedded at build time) for a few tile geometries in one
+//      program, for sm_100a, into a cubin;
+//   3. the cubin is loaded with the driver API in the plan's device context;
+//      the plan's candidates are these kernels, launched by plan_launch like
+//      the ahead-of-time ones (cuLaunchKernel instead of cudaLaunchKernel).
+// Compiled modules are cached per (source, device) for the process lifetime.
+// Host-only plans (SDAG_DEVICE_NONE) generate and compile but do not load, so
+// the generator and the NVRTC build are testable without a GPU.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nvrtc.h>
+
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <sstream>
+#include <string>
+#include <vector>
+
+#include "plan.hpp"
+#include "sweep.cuh"
+
+namespace sdag {
+
+#include "jit_embed.inc"  // kSweepSrc: the text of sweep.cuh
+
+// ---------------------------------------------------------------------------
+// 1. code generation
+// ---------------------------------------------------------------------------
+
+namespace {
+
+std::string num_literal(double v) {
+    char buf[64];
+    std::snprintf(buf, sizeof buf, "%a", v);  // exact
+    return std::string("(") + buf + ")";
+}
+
+struct Gen {
+    const Plan &p;
+    std::vector<bool> written;  // per 3D formal, in program order
+
+    std::string expr(int n) const {
+        const Node &x = p.st.nodes[n];
+        switch (x.kind) {
+        case Node::Num: return num_literal(x.value);
+        case Node::Scalar: return "g.s(" + std::to_string(x.ref) + ")";
+        case Node::Temp: return "t" + std::to_string(x.ref);
+        case Node::Load3: {
+            const int f = x.ref;
+            if (p.in_slot[f] >= 0)
+                return "g.at(" + std::to_string(p.in_slot[f]) + ", " + std::to_string(x.off[0]) + ", " +
+                       std::to_string(x.off[1]) + ", " + std::to_string(x.off[2]) + ")";
+            // a written array, read at offset 0 (analysis rejects shifted reads)
+            if (written[f]) return "v" + std::to_string(p.out_slot[f]);
+            if (p.io_slot[f] >= 0) return "g.io(" + std::to_string(p.io_slot[f]) + ")";
+            throw Error(SDAG_ERR_UNSUPPORTED, "jit: read of an output before it is written");
+        }
+        case Node::Load1: return "g.s1(" + std::to_string(x.ref) + ", " + std::to_string(x.off[0]) + ")";
+        case Node::Neg: return "(-" + expr(x.a) + ")";
+        case Node::Add: return "(" + expr(x.a) + " + " + expr(x.b) + ")";
+        case Node::Sub: return "(" + expr(x.a) + " - " + expr(x.b) + ")";
+        case Node::Mul: return "(" + expr(x.a) + " * " + expr(x.b) + ")";
+        case Node::Div: return "(" + expr(x.a) + " / " + expr(x.b) + ")";
+        }
+        throw Error(SDAG_ERR_UNSUPPORTED, "jit: unknown expression node");
+    }
+};
+
+}  // namespace
+
+// The body struct for the sweep skeleton (interface: sweep.cuh header).
+std::string jit_body_source(const Plan &p, const std::string &sname, int rzr) {
+    const int nin = p.an.n_in, nout = p.an.n_out + p.an.n_inout, nio = p.an.n_inout, n1 = p.n1();
+    std::ostringstream o;
+    o << "struct " << sname << " {\n"
+      << "    static constexpr int NIN = " << nin << ", NOUT = " << nout << ", NIO = " << nio << ", N1D = " << n1
+      << ";\n"
+      << "    static constexpr int RZ = " << p.an.radius[0] << ", RY = " << p.an.radius[1]
+      << ", RX = " << p.an.radius[2] << ", RZR = " << rzr << ";\n"
+      << "    __host__ __device__ static constexpr int axis1d(int a) { return ";
+    for (int f = 0; f < n1; f++) o << "a == " << f << " ? " << p.st.formal(ArgKind::Array1D, f).axis << " : ";
+    o << "2; }\n"
+      << "    template <class G>\n"
+      << "    __device__ __forceinline__ static void eval(const G &g, double (&o)[NOUT]) {\n";
+    for (size_t t = 0; t < p.st.temps.size(); t++) o << "        double t" << t << " = 0.0;\n";
+    for (int m = 0; m < nout; m++) o << "        double v" << m << " = 0.0;\n";
+    Gen g{p, std::vector<bool>(p.n3(), false)};
+    for (const Statement &s : p.st.stmts) {
+        const std::string rhs = g.expr(s.expr);
+        if (s.to_array) {
+            o << "        v" << p.out_slot[s.target] << " = " << rhs << ";  // line " << s.line << "\n";
+            g.written[s.target] = true;
+        } else {
+            o << "        t" << s.target << " = " << rhs << ";  // line " << s.line << "\n";
+        }
+    }
+    for (int m = 0; m < nout; m++) o << "        o[" << m << "] = v" << m << ";\n";
+    o << "    }\n};\n";
+    return o.str();
+}
+
+// ---------------------------------------------------------------------------
+// 2. NVRTC (dlopen'ed, like NCCL in dist.cpp: no link-time dependency)
+// ---------------------------------------------------------------------------
+
+namespace {
+
+struct Nvrtc {
+    decltype(&nvrtcCreateProgram) create = nullptr;
+    decltype(&nvrtcAddNameExpression) add_name = nullptr;
+    decltype(&nvrtcCompileProgram) compile = nullptr;
+    decltype(&nvrtcGetProgramLogSize) log_size = nullptr;
+    decltype(&nvrtcGetProgramLog) log = nullptr;
+    decltype(&nvrtcGetCUBINSize) cubin_size = nullptr;
+    decltype(&nvrtcGetCUBIN) cubin = nullptr;
+    decltype(&nvrtcGetLoweredName) lowered = nullptr;
+    decltype(&nvrtcDestroyProgram) destroy = nullptr;
+    decltype(&nvrtcGetErrorString) errstr = nullptr;
+};
+
+const Nvrtc &nvrtc() {
+    static Nvrtc n = [] {
+        Nvrtc r;
+        void *h = nullptr;
+        for (const char *name : {"libnvrtc.so.12", "libnvrtc.so", "/usr/local/cuda/lib64/libnvrtc.so.12"})
+            if ((h = dlopen(name, RTLD_NOW | RTLD_LOCAL))) break;
+        if (!h) throw Error(SDAG_ERR_UNSUPPORTED, "jit: libnvrtc.so.12 not found (needed for unregistered DAGs)");
+        auto sym = [&](const char *s) {
+            void *f = dlsym(h, s);
+            if (!f) throw Error(SDAG_ERR_UNSUPPORTED, std::string("jit: nvrtc symbol missing: ") + s);
+            return f;
+        };
+        r.create = reinterpret_cast<decltype(r.create)>(sym("nvrtcCreateProgram"));
+        r.add_name = reinterpret_cast<decltype(r.add_name)>(sym("nvrtcAddNameExpression"));
+        r.compile = reinterpret_cast<decltype(r.compile)>(sym("nvrtcCompileProgram"));
+        r.log_size = reinterpret_cast<decltype(r.log_size)>(sym("nvrtcGetProgramLogSize"));
+        r.log = reinterpret_cast<decltype(r.log)>(sym("nvrtcGetProgramLog"));
+        r.cubin_size = reinterpret_cast<decltype(r.cubin_size)>(sym("nvrtcGetCUBINSize"));
+        r.cubin = reinterpret_cast<decltype(r.cubin)>(sym("nvrtcGetCUBIN"));
+        r.lowered = reinterpret_cast<decltype(r.lowered)>(sym("nvrtcGetLoweredName"));
+        r.destroy = reinterpret_cast<decltype(r.destroy)>(sym("nvrtcDestroyProgram"));
+        r.errstr = reinterpret_cast<decltype(r.errstr)>(sym("nvrtcGetErrorString"));
+        return r;
+    }();
+    return n;
+}
+
+// driver entry points through the runtime (libsdag links cudart statically)
+template <class F>
+F drv(const char *name) {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    check_cuda(cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q), name);
+    if (!p || q != cudaDriverEntryPointSuccess) throw Error(SDAG_ERR_CUDA, std::string(name) + " not available");
+    return reinterpret_cast<F>(p);
+}
+
+void check_cu(CUresult r, const char *what) {
+    if (r != CUDA_SUCCESS) throw Error(SDAG_ERR_CUDA, std::string(what) + " failed (CUresult " + std::to_string(r) + ")");
+}
+
+struct Compiled {
+    std::string cubin;
+    std::vector<std::string> lowered;  // per name expression
+    std::string log;
+};
+
+Compiled nvrtc_build(const std::string &src, const std::vector<std::string> &names) {
+    const Nvrtc &N = nvrtc();
+    nvrtcProgram prog;
+    auto ck = [&](nvrtcResult r, const char *what) {
+        if (r != NVRTC_SUCCESS) throw Error(SDAG_ERR_CUDA, std::string("jit: ") + what + ": " + N.errstr(r));
+    };
+    ck(N.create(&prog, src.c_str(), "sdag_jit.cu", 0, nullptr, nullptr), "nvrtcCreateProgram");
+    Compiled c;
+    try {
+        for (const auto &n : names) ck(N.add_name(prog, n.c_str()), "nvrtcAddNameExpression");
+        const char *opts[] = {"-arch=sm_100a", "-std=c++17", "-default-device", "--fmad=true", "-lineinfo",
+                              "--extra-device-vectorization"};
+        const nvrtcResult rc = N.compile(prog, int(sizeof opts / sizeof *opts), opts);
+        size_t ls = 0;
+        N.log_size(prog, &ls);
+        c.log.assign(ls, '\0');
+        if (ls) N.log(prog, &c.log[0]);
+        if (rc != NVRTC_SUCCESS)
+            throw Error(SDAG_ERR_UNSUPPORTED, "jit: NVRTC compile failed: " + std::string(N.errstr(rc)) + "\n" + c.log);
+        size_t cs = 0;
+        ck(N.cubin_size(prog, &cs), "nvrtcGetCUBINSize");
+        c.cubin.assign(cs, '\0');
+        ck(N.cubin(prog, &c.cubin[0]), "nvrtcGetCUBIN");
+        for (const auto &n : names) {
+            const char *l = nullptr;
+            ck(N.lowered(prog, n.c_str(), &l), "nvrtcGetLoweredName");
+            c.lowered.push_back(l);
+        }
+    } catch (...) {
+        N.destroy(&prog);
+        throw;
+    }
+    N.destroy(&prog);
+    return c;
+}
+
+struct Module {
+    CUmodule mod = nullptr;
+    std::vector<CUfunction> fns;
+};
+
+std::mutex g_jit_mu;
+std::map<std::string, Compiled> g_compiled;            // source -> cubin
+std::map<std::pair<std::string, int>, Module> g_mods;  // (source, device) -> module
+
+struct Geom {
+    int tx, ty, ux, uy, pf;
+};
+
+}  // namespace
+
+// ---------------------------------------------------------------------------
+// 3. plan integration
+// ---------------------------------------------------------------------------
+
+// Fill p->jit_descs / p->cands with NVRTC-compiled skeleton kernels for the
+// plan's DAG.  Throws UNSUPPORTED when the DAG exceeds the skeleton's limits.
+void jit_build_candidates(Plan *p) {
+    using namespace dev;
+    const int nin = p->an.n_in, nout = p->an.n_out + p->an.n_inout, nio = p->an.n_inout, n1 = p->n1();
+    if (nin < 1 || nin > MAXIN || nout > MAXOUT || nio > MAXIO || n1 > MAX1D || p->ns() > MAXS)
+        throw Error(SDAG_ERR_UNSUPPORTED,
+                    "jit: DAG outside the sweep skeleton's limits (1.." + std::to_string(MAXIN) + " inputs, <= " +
+                        std::to_string(MAXOUT) + " outputs, <= " + std::to_string(MAXIO) + " inouts, <= " +
+                        std::to_string(MAX1D) + " 1D arrays, <= " + std::to_string(MAXS) + " scalars)");
+    const int RZ = p->an.radius[0], RY = p->an.radius[1], RX = p->an.radius[2];
+
+    // tile geometries, preference order (the generic skeleton's best shapes on
+    // the registered DAGs: tools/perf_sweep.py); smem decides RZR
+    const Geom geoms[] = {{32, 16, 1, 2, 1}, {64, 8, 1, 1, 1}, {16, 16, 1, 1, 1}};
+    struct Cand {
+        Geom g;
+        int rzr;
+        bool tma;
+        int smem;
+        std::string name;
+    };
+    std::vector<Cand> cs;
+    bool need_r0 = false, need_full = false;
+    for (const Geom &g : geoms) {
+        const int px = g.tx + 2 * RX, py = g.ty + 2 * RY;
+        if (px > 256 || py > 256) continue;
+        const int plane_al = ((px * py * 8 + 127) / 128) * 128 / 8;
+        for (int rzr : {RZ, 0}) {
+            const int ns = 2 * rzr + 1 + g.pf;
+            const int smem = ns * nin * plane_al * 8 + ns * 8;
+            if (smem > 227 * 1024) continue;
+            (rzr == RZ ? need_full : need_r0) = true;
+            for (bool tma : {true, false}) cs.push_back({g, rzr, tma, smem, ""});
+            break;
+        }
+    }
+    if (cs.empty()) throw Error(SDAG_ERR_UNSUPPORTED, "jit: no tile geometry fits 227 KB of shared memory");
+
+    std::ostringstream src;
+    src << "// generated by sdag jit.cpp for stencil '" << p->st.name << "'\n" << kSweepSrc << "\n"
+        << "namespace sdag {\nnamespace dev {\n";
+    if (need_full) src << jit_body_source(*p, "JitBody", RZ);
+    if (need_r0 && RZ > 0) src << jit_body_source(*p, "JitBodyR0", 0);
+    if (need_r0 && RZ == 0 && !need_full) src << jit_body_source(*p, "JitBody", 0);
+    src << "}  // namespace dev\n}  // namespace sdag\n";
+    std::vector<std::string> names;
+    for (Cand &c : cs) {
+        const char *body = (c.rzr == RZ) ? "JitBody" : "JitBodyR0";
+        char buf[160];
+        std::snprintf(buf, sizeof buf, "sdag::dev::sdag_sweep<sdag::dev::%s, %d, %d, %d, %d, %d, %s>", body, c.g.tx,
+                      c.g.ty, c.g.ux, c.g.uy, c.g.pf, c.tma ? "true" : "false");
+        names.push_back(buf);
+        std::snprintf(buf, sizeof buf, "jit_%s_%dx%d_u%dx%d_pf%d%s", c.tma ? "tma" : "lsu", c.g.tx, c.g.ty, c.g.ux,
+                      c.g.uy, c.g.pf, (c.rzr == RZ) ? "" : "_r0");
+        c.name = buf;
+    }
+    const std::string key = src.str();
+
+    std::lock_guard<std::mutex> lk(g_jit_mu);
+    auto it = g_compiled.find(key);
+    if (it == g_compiled.end()) it = g_compiled.emplace(key, nvrtc_build(key, names)).first;
+    const Compiled &cc = it->second;
+    p->jit_source = key;
+
+    std::vector<CUfunction> fns(cs.size(), nullptr);
+    if (!p->host_only) {
+        auto mk = std::make_pair(key, p->device);
+        auto mt = g_mods.find(mk);
+        if (mt == g_mods.end()) {
+            int prev = -1;
+            check_cuda(cudaGetDevice(&prev), "cudaGetDevice");
+            check_cuda(cudaSetDevice(p->device), "cudaSetDevice");
+            check_cuda(cudaFree(nullptr), "context init");  // make the primary context current
+            using LoadT = decltype(&cuModuleLoadData);
+            using GetT = decltype(&cuModuleGetFunction);
+            Module m;
+            CUresult r = drv<LoadT>("cuModuleLoadData")(&m.mod, cc.cubin.data());
+            if (r == CUDA_SUCCESS)
+                for (const auto &l : cc.lowered) {
+                    CUfunction f = nullptr;
+                    r = drv<GetT>("cuModuleGetFunction")(&f, m.mod, l.c_str());
+                    if (r != CUDA_SUCCESS) break;
+                    m.fns.push_back(f);
+                }
+            cudaSetDevice(prev);
+            check_cu(r, "jit: cuModuleLoadData/cuModuleGetFunction");
+            mt = g_mods.emplace(mk, m).first;
+        }
+        fns = mt->second.fns;
+    }
+    for (size_t q = 0; q < cs.size(); q++) {
+        const Cand &c = cs[q];
+        auto d = std::make_unique<KernelDesc>();
+        d->dag = "(jit)";
+        d->variant = c.name;
+        d->fn = nullptr;
+        d->cufn = fns[q];
+        d->threads = (c.g.tx / c.g.ux) * (c.g.ty / c.g.uy);
+        d->smem = c.smem;
+        d->tx = c.g.tx;
+        d->ty = c.g.ty;
+        d->ux = c.g.ux;
+        d->uy = c.g.uy;
+        d->pf = c.g.pf;
+        d->tma = c.tma;
+        d->nin = nin;
+        d->nout = nout;
+        d->nio = nio;
+        d->n1d = n1;
+        d->rz = RZ;
+        d->ry = RY;
+        d->rx = RX;
+        d->rzr = c.rzr;
+        d->prio = int(q / 2) + (c.tma ? 0 : 100);
+        p->jit_descs.push_back(std::move(d));
+    }
+}
+
+// launch / occupancy of a JIT kernel (driver API)
+void jit_launch(const KernelDesc &k, dim3 grid, void **args, cudaStream_t stream) {
+    using AttrT = decltype(&cuFuncSetAttribute);
+    using LaunchT = decltype(&cuLaunchKernel);
+    static AttrT set_attr = drv<AttrT>("cuFuncSetAttribute");
+    static LaunchT launch = drv<LaunchT>("cuLaunchKernel");
+    CUfunction f = static_cast<CUfunction>(k.cufn);
+    check_cu(set_attr(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, k.smem), "jit: cuFuncSetAttribute");
+    check_cu(launch(f, grid.x, grid.y, grid.z, k.threads, 1, 1, unsigned(k.smem), reinterpret_cast<CUstream>(stream),
+                    args, nullptr),
+             "jit: cuLaunchKernel");
+}
+
+int jit_occupancy(const KernelDesc &k) {
+    using OccT = decltype(&cuOccupancyMaxActiveBlocksPerMultiprocessor);
+    static OccT occ = drv<OccT>("cuOccupancyMaxActiveBlocksPerMultiprocessor");
+    int n = 0;
+    if (occ(&n, static_cast<CUfunction>(k.cufn), k.threads, size_t(k.smem)) != CUDA_SUCCESS) return 0;
+    return n;
+}
+
+}  // namespace sdag

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <map>
+#include <memory>
 #include <mutex>
 #include <string>
 #include <tuple>
@@ -43,6 +44,8 @@ struct Plan {
     std::vector<const KernelDesc *> fused;  // multi-sweep kernels for apply_iterated (tsteps > 1)
     double fcost[8] = {0};                  // f(x): relative cost of an x-sweep launch (deep tuning)
     bool fusion = true;                     // use fused kernels in apply_iterated
+    std::vector<std::unique_ptr<KernelDesc>> jit_descs;  // NVRTC kernels of an unregistered DAG (NEXT-4)
+    std::string jit_source;                 // their generated source (sdag_plan_describe shows the body)
     int chosen = -1;                        // index into cands
     std::string describe_text;
 
@@ -77,6 +80,11 @@ void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int
 void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int n1, const double *s, int ns,
                 cudaStream_t stream, int64_t *h2d, int64_t *d2h);
 void check_cuda(cudaError_t e, const char *what);
+// jit.cu (NEXT-4)
+std::string jit_body_source(const Plan &p, const std::string &sname, int rzr);
+void jit_build_candidates(Plan *p);
+void jit_launch(const KernelDesc &k, dim3 grid, void **args, cudaStream_t stream);
+int jit_occupancy(const KernelDesc &k);
 
 // process-wide launch counter
 void count_launch();

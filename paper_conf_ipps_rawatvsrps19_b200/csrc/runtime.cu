@@ -123,7 +123,10 @@ static CUtensorMap tmap_for(Plan *p, const double *ptr, int64_t nx, int64_t ny, 
 // ---------------------------------------------------------------------------
 
 static int occupancy_of(const Plan *p, const KernelDesc &k) {
-    if (!p->host_only) {
+    if (!p->host_only && k.cufn) {
+        const int n = jit_occupancy(k);
+        if (n > 0) return n;
+    } else if (!p->host_only) {
         int n = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k.fn, k.threads, k.smem) == cudaSuccess && n > 0)
             return n;
@@ -238,7 +241,7 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *
     const int nlaunch = k.fission ? int(k.fission_fns.size()) : 1;
     for (int q = 0; q < nlaunch; q++) {
         const void *fn = k.fission ? k.fission_fns[q] : k.fn;
-        {
+        if (!k.cufn) {
             std::lock_guard<std::mutex> g(attr_mu);
             int &d = attr_done[fn];
             if (d < k.smem) {
@@ -255,7 +258,10 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *
         dim3 grid(L.tiles_x, L.tiles_y, L.nchunk * batch);
         if (grid.z > 65535 || grid.y > 65535) throw Error(SDAG_ERR_DOMAIN, "grid too large (batch x chunks > 65535)");
         void *args[] = {&Aq};
-        check_cuda(cudaLaunchKernel(fn, grid, dim3(k.threads), args, size_t(k.smem), stream), "sweep launch");
+        if (k.cufn)
+            jit_launch(k, grid, args, stream);
+        else
+            check_cuda(cudaLaunchKernel(fn, grid, dim3(k.threads), args, size_t(k.smem), stream), "sweep launch");
         count_launch();
     }
 }
@@ -509,23 +515,37 @@ Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_pla
     }
 
     std::ostringstream d;
-    d << "stencil '" << p->st.name << "' -> dag '" << (p->reg ? p->reg->name : std::string("(unregistered)"))
+    // NEXT-4: unregistered DAGs (or force_variant "jit...") are code-generated and
+    // compiled with NVRTC into the generic skeleton (jit.cu); host-only plans of
+    // unregistered DAGs stay analysis-only unless "jit" is forced
+    const bool forced_jit = p->force_variant.rfind("jit", 0) == 0;
+    const bool use_jit = forced_jit || (!p->reg && !p->host_only);
+    if (use_jit) {
+        p->reg = nullptr;
+        p->extra_scalars.clear();
+    }
+    d << "stencil '" << p->st.name << "' -> dag '"
+      << (p->reg ? p->reg->name : std::string(use_jit ? "(jit)" : "(unregistered)"))
       << "'\n"
       << "  radius (z,y,x) = (" << p->an.radius[0] << "," << p->an.radius[1] << "," << p->an.radius[2] << ")"
       << "  flops/pt = " << p->an.flops_per_point << "  bytes/pt = " << p->bytes_per_point()
       << "  IO arrays = " << p->an.n_io_arrays << "  homogenizable(z) = " << (p->an.homogenizable_z ? "yes" : "no");
-    if (!p->reg) {
-        // analysis-only plans are allowed host-only; a device plan needs a kernel
-        if (!p->host_only)
-            throw Error(SDAG_ERR_UNSUPPORTED, "no sm_100a kernel is registered for this stencil DAG (registered: " +
-                                                  registry_names() + "); arbitrary DAG code generation is NEXT-4");
-        d << "\n  no registered sm_100a body (analysis only)";
+    if (!p->reg && !use_jit) {
+        // analysis-only host plan
+        d << "\n  no registered sm_100a body (analysis only; force_variant \"jit\" compiles one)";
         p->describe_text = d.str();
         return p.release();
     }
 
     // candidates: kernels of this DAG, TMA variants only when nx is even
+    if (use_jit) {
+        jit_build_candidates(p.get());
+        for (auto &k : p->jit_descs)
+            if (!k->tma || p->dims[2] % 2 == 0) p->cands.push_back(k.get());
+        if (p->force_variant == "jit") p->force_variant.clear();
+    }
     for (const KernelDesc &k : kernel_table()) {
+        if (use_jit) break;
         if (k.dag != p->reg->name) continue;
         if (k.tma && p->dims[2] % 2 != 0) continue;
         if (k.smem > 227 * 1024) continue;
@@ -575,6 +595,8 @@ Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_pla
         for (int x = 1; x < 8; x++)
             if (p->fcost[x] > 0.0) d << " f(" << x << ")=" << p->fcost[x];
     }
+    if (!p->jit_descs.empty())
+        d << "\n  jit body (NVRTC, sm_100a, into the sweep.cuh skeleton):\n" << jit_body_source(*p, "JitBody", p->an.radius[0]);
     p->describe_text = d.str();
     return p.release();
 }
@@ -683,7 +705,7 @@ void plan_fill_info(Plan *p, sdag_plan_info *info) {
     info->oi_paper = p->an.n_io_arrays ? p->an.flops_per_point / (8.0 * p->an.n_io_arrays) : 0.0;
     info->n_kernels = (!p->cands.empty() && p->kernel().fission) ? int(p->kernel().fission_fns.size()) : 1;
     info->n_variants = int(p->cands.size());
-    info->dag = p->reg ? p->reg->name.c_str() : "";
+    info->dag = p->reg ? p->reg->name.c_str() : (p->jit_descs.empty() ? "" : "(jit)");
     info->variant = p->cands.empty() ? "" : p->kernel().variant.c_str();
     if (p->cands.empty()) info->n_kernels = 0;
 }

@@ -31,9 +31,21 @@
 // with g.at(arr, dz, dy, dx), g.io(m), g.s1(arr, off), g.s(n).
 #pragma once
 
+#ifdef __CUDACC_RTC__
+// NVRTC (jit.cu, NEXT-4): no host headers; the few types the skeleton needs
+typedef unsigned int uint32_t;
+typedef int int32_t;
+typedef unsigned long long uint64_t;
+typedef long long int64_t;
+typedef unsigned long long uintptr_t;
+struct alignas(64) CUtensorMap {
+    unsigned long long opaque[16];
+};
+#else
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#endif
 
 namespace sdag {
 namespace dev {
