@@ -22,23 +22,27 @@
 namespace sdag {
 namespace dev {
 
-template <int GX, int GY, int UY, int PF>
+template <int GX, int GY, int UY, int PF, int UX = 2>
 struct Fuse2Geo {
     static constexpr int ML = 2;                 // box x margin (region - 2): 16-B alignment
-    static constexpr int NTX = GX / 2, NTY = GY / UY, THREADS = NTX * NTY, NWARPS = (THREADS + 31) / 32;
+    static constexpr int NTX = GX / UX, NTY = GY / UY, THREADS = NTX * NTY, NWARPS = (THREADS + 31) / 32;
     static constexpr int PX = GX + 4, PY = GY + 2, PLANE = PX * PY;  // input box / S1 plane layout
     static constexpr int PLANE_AL = ((PLANE * 8 + 127) / 128) * 128 / 8;
     static constexpr int NS = 1 + PF;
     static constexpr int SMEM = (NS + 2) * PLANE_AL * 8 + 2 * NS * 8;
-    static_assert(GX % 2 == 0 && GY % UY == 0, "region");
+    static constexpr int NW = UX + 4;            // row window [cx, cx+UX+4) in smem columns (16-B aligned)
+    static_assert((UX == 2 || UX == 4) && GX % UX == 0 && GY % UY == 0, "region");
     static_assert(PX <= 256 && PY <= 256, "TMA box");
 };
 
-template <int GX, int GY, int UY, int PF, int MINB = 1>
-__global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF>::THREADS, MINB)
+// UX = 2 or 4 output columns per thread: the row window of a UX-wide patch is
+// UX+4 doubles read with (UX+4)/2 128-bit loads, so UX = 4 cuts the fold's
+// shared-memory reads per point from 1.5 to 1 LDS.128 per row.
+template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2>
+__global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX>::THREADS, MINB)
     sdag_box27x2(const __grid_constant__ SweepArgs a) {
-    using G = Fuse2Geo<GX, GY, UY, PF>;
-    constexpr int PX = G::PX, NS = G::NS, PAL = G::PLANE_AL, ML = G::ML;
+    using G = Fuse2Geo<GX, GY, UY, PF, UX>;
+    constexpr int PX = G::PX, NS = G::NS, PAL = G::PLANE_AL, ML = G::ML, NW = G::NW;
     constexpr int TX = GX - 2, TY = GY - 2;  // output tile
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -61,13 +65,13 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF>::THREADS, MINB)
 
     const int t = threadIdx.x;
     const int lx = t % G::NTX, ly = t / G::NTX;
-    const int cx = 2 * lx, cy = UY * ly;  // patch origin in region coordinates
+    const int cx = UX * lx, cy = UY * ly;  // patch origin in region coordinates
 
     auto issue = [&](int p) {
-        const int slot = (p - p0) % NS;
+        const int slot = unsigned(p - p0) % NS;
         if (t == 0) {
             const int prev = p - NS;
-            if (prev >= p0) mbar_wait(&empty[slot], ((prev - p0) / NS) & 1);
+            if (prev >= p0) mbar_wait(&empty[slot], (unsigned(prev - p0) / NS) & 1);
             mbar_expect_tx(&full[slot], uint32_t(G::PLANE * 8));
             tma_load_3d(ring + slot * PAL, &a.tmap[0], &full[slot], rx0 - ML, ry0 - 1, int(zbase + p));
         }
@@ -86,34 +90,37 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF>::THREADS, MINB)
     const double w0 = a.s[0], w1 = a.s[1], w2 = a.s[2], w3 = a.s[3], nu = a.s[4];
 
     // region point (cy+py, cx+px) -> global (ry0+cy+py, rx0+cx+px); x/y ring flags
-    bool ringxy[UY][2];
+    bool ringxy[UY][UX];
 #pragma unroll
     for (int py = 0; py < UY; py++)
 #pragma unroll
-        for (int px = 0; px < 2; px++) {
+        for (int px = 0; px < UX; px++) {
             const int gy = ry0 + cy + py, gx = rx0 + cx + px;
             ringxy[py][px] = gy <= 0 || gy >= ny - 1 || gx <= 0 || gx >= nx - 1;
         }
     // outputs: tile points strictly inside the region and inside the interior
     const int gi = rx0 + cx;
-    const bool out0 = cx >= 1 && cx <= TX && gi >= a.xmin && gi < a.hi[2];
-    const bool out1 = cx + 1 >= 1 && cx + 1 <= TX && gi + 1 >= a.xmin && gi + 1 < a.hi[2];
+    bool outm[UX];
+#pragma unroll
+    for (int px = 0; px < UX; px++)
+        outm[px] = cx + px >= 1 && cx + px <= TX && gi + px >= a.xmin && gi + px < a.hi[2];
+    const bool vec_ok = (a.nx % 2 == 0) && ((reinterpret_cast<uintptr_t>(a.out[0]) & 15) == 0) && (gi % 2 == 0);
 
-    double T1[UY][2], U1[UY][2], A1[UY][2];  // sweep-1 retimed state
-    double T2[UY][2], U2[UY][2], A2[UY][2];  // sweep-2 retimed state
+    double T1[UY][UX], U1[UY][UX], A1[UY][UX];  // sweep-1 retimed state
+    double T2[UY][UX], U2[UY][UX], A2[UY][UX];  // sweep-2 retimed state
 #pragma unroll
     for (int py = 0; py < UY; py++)
 #pragma unroll
-        for (int px = 0; px < 2; px++) T1[py][px] = U1[py][px] = A1[py][px] = T2[py][px] = U2[py][px] = A2[py][px] = 0.0;
+        for (int px = 0; px < UX; px++) T1[py][px] = U1[py][px] = A1[py][px] = T2[py][px] = U2[py][px] = A2[py][px] = 0.0;
 
     // in-plane partial sums -> (c, u) of one plane at the patch points
-    auto fold = [&](const double *pl, double (&cc)[UY][2], double (&uu)[UY][2], double (&s0v)[UY][2]) {
-        double w[UY + 2][6];
+    auto fold = [&](const double *pl, double (&cc)[UY][UX], double (&uu)[UY][UX], double (&s0v)[UY][UX]) {
+        double w[UY + 2][NW];
 #pragma unroll
         for (int r = 0; r < UY + 2; r++) {
             const double *rp = pl + (cy + r) * PX + cx;
 #pragma unroll
-            for (int c = 0; c < 3; c++) {
+            for (int c = 0; c < NW / 2; c++) {
                 const double2 v = *reinterpret_cast<const double2 *>(rp + 2 * c);
                 w[r][2 * c] = v.x;
                 w[r][2 * c + 1] = v.y;
@@ -122,7 +129,7 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF>::THREADS, MINB)
 #pragma unroll
         for (int py = 0; py < UY; py++)
 #pragma unroll
-            for (int px = 0; px < 2; px++) {
+            for (int px = 0; px < UX; px++) {
                 const int c = ML + px;
                 const double s0 = w[py + 1][c];
                 const double s1 = (w[py + 1][c - 1] + w[py + 1][c + 1]) + (w[py][c] + w[py + 2][c]);
@@ -135,28 +142,31 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF>::THREADS, MINB)
 
     for (int p = p0; p <= plast; p++) {
         if (p + PF <= plast) issue(p + PF);
-        mbar_wait(&full[(p - p0) % NS], ((p - p0) / NS) & 1);
+        mbar_wait(&full[unsigned(p - p0) % NS], (unsigned(p - p0) / NS) & 1);
         // ---- sweep 1: input plane p completes sweep-1 plane j = p-1 on the region ----
-        double cc[UY][2], uu[UY][2], s0[UY][2];
-        fold(ring + ((p - p0) % NS) * PAL, cc, uu, s0);
+        double cc[UY][UX], uu[UY][UX], s0[UY][UX];
+        fold(ring + (unsigned(p - p0) % NS) * PAL, cc, uu, s0);
         __syncwarp();
         if ((t & 31) == 0)
-            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[(p - p0) % NS])) : "memory");
+            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[unsigned(p - p0) % NS]))
+                         : "memory");
         const int j = p - 1;
         const bool zring = j <= 0 || j >= nz - 1;
         double *s1 = s1buf + (j & 1) * PAL;
 #pragma unroll
         for (int py = 0; py < UY; py++) {
-            double v[2];
+            double v[UX];
 #pragma unroll
-            for (int px = 0; px < 2; px++) {
+            for (int px = 0; px < UX; px++) {
                 v[px] = fma(nu, T1[py][px] + uu[py][px], A1[py][px]);
                 if (zring || ringxy[py][px]) v[px] = A1[py][px];  // ring: not updated by sweep 1
                 T1[py][px] = U1[py][px] + cc[py][px];
                 U1[py][px] = uu[py][px];
                 A1[py][px] = s0[py][px];
             }
-            *reinterpret_cast<double2 *>(s1 + (cy + py + 1) * PX + cx + ML) = make_double2(v[0], v[1]);
+#pragma unroll
+            for (int px = 0; px < UX; px += 2)
+                *reinterpret_cast<double2 *>(s1 + (cy + py + 1) * PX + cx + ML + px) = make_double2(v[px], v[px + 1]);
         }
         __syncthreads();  // sweep-1 plane j is complete in shared memory
         if (j < kb - 1) continue;  // sweep-2 state starts at sweep-1 plane kb-1
@@ -166,9 +176,9 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF>::THREADS, MINB)
         double *o = a.out[0] + ((zbase + k) * a.ny + (ry0 + cy)) * a.nx + gi;
 #pragma unroll
         for (int py = 0; py < UY; py++) {
-            double res[2];
+            double res[UX];
 #pragma unroll
-            for (int px = 0; px < 2; px++) {
+            for (int px = 0; px < UX; px++) {
                 res[px] = fma(nu, T2[py][px] + uu[py][px], A2[py][px]);
                 T2[py][px] = U2[py][px] + cc[py][px];
                 U2[py][px] = uu[py][px];
@@ -176,8 +186,15 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF>::THREADS, MINB)
             }
             const int ry = cy + py, gj = ry0 + ry;
             if (k >= kb && ry >= 1 && ry <= TY && gj < a.hi[1]) {
-                if (out0) __stcs(o, res[0]);
-                if (out1) __stcs(o + 1, res[1]);
+#pragma unroll
+                for (int px = 0; px < UX; px += 2) {
+                    if (vec_ok && outm[px] && outm[px + 1]) {
+                        __stcs(reinterpret_cast<double2 *>(o + px), make_double2(res[px], res[px + 1]));
+                    } else {
+                        if (outm[px]) __stcs(o + px, res[px]);
+                        if (outm[px + 1]) __stcs(o + px + 1, res[px + 1]);
+                    }
+                }
             }
             o += a.nx;
         }

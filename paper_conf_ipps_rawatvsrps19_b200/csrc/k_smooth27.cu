@@ -17,5 +17,6 @@ void add_kernels_smooth27(std::vector<KernelDesc> &v) {
     v.push_back(make_fuse2_desc<128, 16, 4, 2>("smooth27", 22));
     v.push_back(make_fuse2_desc<64, 32, 2, 2>("smooth27", 23));
     v.push_back(make_fuse2_desc<128, 16, 2, 2>("smooth27", 24));
+    v.push_back(make_fuse2_desc<64, 16, 2, 2, 1, 4>("smooth27", 25));  // 4-wide patch: bank-conflicted, kept for comparison
 }
 }  // namespace sdag

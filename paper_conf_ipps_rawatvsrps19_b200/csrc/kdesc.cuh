@@ -199,23 +199,23 @@ KernelDesc make_star2_desc(const char *dag, int prio) {
     v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, QM, 1>(DAG, PRIO))
 
 // two fused sweeps of the 27-point smoother (fuse2.cuh), TMA only
-template <int GX, int GY, int UY, int PF, int MINB = 1>
+template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2>
 KernelDesc make_fuse2_desc(const char *dag, int prio) {
-    using G = dev::Fuse2Geo<GX, GY, UY, PF>;
+    using G = dev::Fuse2Geo<GX, GY, UY, PF, UX>;
     KernelDesc d;
     d.dag = dag;
     char buf[96];
     if (MINB > 1)
-        std::snprintf(buf, sizeof buf, "fuse2_tma_%dx%d_u2x%d_pf%d_mb%d", GX - 2, GY - 2, UY, PF, MINB);
+        std::snprintf(buf, sizeof buf, "fuse2_tma_%dx%d_u%dx%d_pf%d_mb%d", GX - 2, GY - 2, UX, UY, PF, MINB);
     else
-        std::snprintf(buf, sizeof buf, "fuse2_tma_%dx%d_u2x%d_pf%d", GX - 2, GY - 2, UY, PF);
+        std::snprintf(buf, sizeof buf, "fuse2_tma_%dx%d_u%dx%d_pf%d", GX - 2, GY - 2, UX, UY, PF);
     d.variant = buf;
-    d.fn = reinterpret_cast<const void *>(&dev::sdag_box27x2<GX, GY, UY, PF, MINB>);
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_box27x2<GX, GY, UY, PF, MINB, UX>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = GX - 2;
     d.ty = GY - 2;
-    d.ux = 2;
+    d.ux = UX;
     d.uy = UY;
     d.pf = PF;
     d.tma = true;
