@@ -87,9 +87,14 @@ typedef struct sdag_plan_opts {
     int32_t fusion;            /* sdag_apply_iterated: 1 = fuse sweeps where a fused kernel
                                   exists (temporal fusion), 0 = one launch
                                   per sweep                                               */
+    int32_t time_tile;         /* sdag_dist_*: ghost depth H = R_z x time_tile (1..7), so a
+                                  fused launch of up to time_tile sweeps runs between two
+                                  halo exchanges (communication-avoiding temporal fusion,
+                                  SURVEY 8(f) NEXT-1); 1 = exchange every sweep         */
 } sdag_plan_opts;
 
-/* Fills `o` with the defaults {order=-1, device=CURRENT, tune=0, batch=1, NULL, fusion=1}. */
+/* Fills `o` with the defaults {order=-1, device=CURRENT, tune=0, batch=1, NULL, fusion=1,
+ * time_tile=1}. */
 void sdag_plan_opts_init(sdag_plan_opts *o);
 
 typedef struct sdag_plan_info {
@@ -197,6 +202,16 @@ sdag_status sdag_slab_partition(int64_t global_nz, int32_t rz, int32_t nranks, i
  * same for the upper neighbour (-1 = no such neighbour), out[4] = rz. */
 sdag_status sdag_slab_halo(int64_t global_nz, int32_t rz, int32_t nranks, int32_t rank, int64_t out[5]);
 
+/* As sdag_slab_partition / sdag_slab_halo for a ghost depth H = rz * time_tile:
+ * out[7] = H; local plane 0 is global plane out[0] - H.  The halo schedule of
+ * one exchange of `planes` (0..H) planes: ranks send their `planes` owned
+ * planes next to each neighbour and receive the same number into the ghost
+ * planes adjacent to their owned range.  Error DOMAIN if a rank would own < H. */
+sdag_status sdag_slab_partition2(int64_t global_nz, int32_t rz, int32_t time_tile, int32_t nranks, int32_t rank,
+                                 int64_t out[8]);
+sdag_status sdag_slab_halo2(int64_t global_nz, int32_t rz, int32_t time_tile, int32_t nranks, int32_t rank,
+                            int32_t planes, int64_t out[5]);
+
 /* NCCL bootstrap through the same libnccl.so.2 torch loads (dlopen).
  * unique id: 128 bytes, broadcast by the caller (e.g. torch.distributed). */
 sdag_status sdag_nccl_get_unique_id(uint8_t id[128]);
@@ -220,7 +235,12 @@ sdag_plan sdag_dist_local_plan(sdag_dist d);
 sdag_status sdag_dist_apply(sdag_dist d, double *const *arrays3d, int32_t n3d, const double *const *arrays1d,
                             int32_t n1d, const double *scalars, int32_t nscalars, sdag_stream compute,
                             sdag_stream comm);
-/* T sweeps, ping-pong, exchange every sweep (1 in -> 1 out plans). Result in buf[T&1]. */
+/* T sweeps, ping-pong (1 in -> 1 out plans), result in buf[T&1].  With
+ * opts.time_tile = t > 1 and a fused kernel (opts.fusion), the sweeps are
+ * scheduled as fused launches of up to t sweeps (the apply_iterated DP), each
+ * preceded by ONE exchange of x R_z planes (x = its sweeps): 1/x of the
+ * exchanges; planes next to the ghosts are recomputed redundantly inside the
+ * launch.  Bit-identical to the single-GPU sdag_apply_iterated schedule. */
 sdag_status sdag_dist_apply_iterated(sdag_dist d, double *buf0, double *buf1, int32_t T, const double *scalars,
                                      int32_t nscalars, sdag_stream compute, sdag_stream comm);
 void sdag_dist_destroy(sdag_dist d);

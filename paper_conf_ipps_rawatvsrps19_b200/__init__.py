@@ -21,7 +21,7 @@ import os
 from . import _capi
 from ._capi import PlanInfo, PlanOpts, SDAG_DEVICE_CURRENT, SDAG_DEVICE_NONE
 
-__all__ = ["Plan", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "nccl_unique_id",
+__all__ = ["Plan", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "slab_partition2", "slab_halo2", "nccl_unique_id",
            "nccl_comm_create", "nccl_comm_destroy", "launch_count", "fp64_peak", "version", "SPEC_DIR"]
 
 SPEC_DIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "specs")
@@ -67,7 +67,7 @@ def _scal(s):
     return (ctypes.c_double * max(1, len(s)))(*s), len(s)
 
 
-def _opts(order=-1, device=None, tune=False, batch=1, variant=None, fusion=True):
+def _opts(order=-1, device=None, tune=False, batch=1, variant=None, fusion=True, time_tile=1):
     o = PlanOpts()
     _capi.lib().sdag_plan_opts_init(ctypes.byref(o))
     o.order = int(order)
@@ -87,6 +87,7 @@ def _opts(order=-1, device=None, tune=False, batch=1, variant=None, fusion=True)
     o.batch = int(batch)
     o.force_variant = variant.encode() if variant else None
     o.fusion = 1 if fusion else 0
+    o.time_tile = int(time_tile)
     return o
 
 
@@ -233,6 +234,21 @@ def slab_partition(global_nz: int, rz: int, nranks: int, rank: int) -> dict:
     return dict(zip(keys, list(out)))
 
 
+def slab_partition2(global_nz: int, rz: int, time_tile: int, nranks: int, rank: int) -> dict:
+    """slab_partition with ghost depth H = rz * time_tile (key "halo")."""
+    out = (ctypes.c_int64 * 8)()
+    _check(_capi.lib().sdag_slab_partition2(int(global_nz), int(rz), int(time_tile), int(nranks), int(rank), out))
+    keys = ("z0", "nz_own", "nz_alloc", "k_lo", "k_hi", "has_lower", "has_upper", "halo")
+    return dict(zip(keys, list(out)))
+
+
+def slab_halo2(global_nz: int, rz: int, time_tile: int, nranks: int, rank: int, planes: int) -> dict:
+    out = (ctypes.c_int64 * 5)()
+    _check(_capi.lib().sdag_slab_halo2(int(global_nz), int(rz), int(time_tile), int(nranks), int(rank), int(planes),
+                                        out))
+    return dict(zip(("lo_send", "lo_recv", "up_send", "up_recv", "planes"), list(out)))
+
+
 def slab_halo(global_nz: int, rz: int, nranks: int, rank: int) -> dict:
     out = (ctypes.c_int64 * 5)()
     _check(_capi.lib().sdag_slab_halo(int(global_nz), int(rz), int(nranks), int(rank), out))
@@ -258,11 +274,12 @@ def nccl_comm_destroy(comm: int):
 class Dist:
     """This rank's z-slab of a global stencil problem (a7)."""
 
-    def __init__(self, spec, global_dims, rank, nranks, comm=None, order=-1, device=None, tune=False, variant=None):
+    def __init__(self, spec, global_dims, rank, nranks, comm=None, order=-1, device=None, tune=False, variant=None,
+                 fusion=True, time_tile=1):
         self._L = _capi.lib()
         self._h = ctypes.c_void_p()
         d = (ctypes.c_int64 * 3)(*[int(x) for x in global_dims])
-        o = _opts(order, device, tune, 1, variant)
+        o = _opts(order, device, tune, 1, variant, fusion, time_tile)
         _check(self._L.sdag_dist_create(spec.encode(), d, ctypes.byref(o), int(rank), int(nranks),
                                         ctypes.c_void_p(comm or 0), ctypes.byref(self._h)))
         self.rank, self.nranks = rank, nranks

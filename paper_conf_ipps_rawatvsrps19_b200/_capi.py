@@ -18,7 +18,7 @@ c_dblp = ctypes.POINTER(c_dbl)
 
 class PlanOpts(ctypes.Structure):
     _fields_ = [("order", c_i32), ("device", c_i32), ("tune", c_i32), ("batch", c_i32),
-                ("force_variant", c_char_p), ("fusion", c_i32)]
+                ("force_variant", c_char_p), ("fusion", c_i32), ("time_tile", c_i32)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -66,6 +66,8 @@ def lib():
                                          ctypes.POINTER(c_i32), c_dblp]),
             "sdag_slab_partition": (S, [c_i64, c_i32, c_i32, c_i32, c_i64p]),
             "sdag_slab_halo": (S, [c_i64, c_i32, c_i32, c_i32, c_i64p]),
+            "sdag_slab_partition2": (S, [c_i64, c_i32, c_i32, c_i32, c_i32, c_i64p]),
+            "sdag_slab_halo2": (S, [c_i64, c_i32, c_i32, c_i32, c_i32, c_i32, c_i64p]),
             "sdag_nccl_get_unique_id": (S, [ctypes.c_char_p]),
             "sdag_nccl_comm_create": (S, [ctypes.c_char_p, c_i32, c_i32, c_i32, ctypes.POINTER(c_void_p)]),
             "sdag_nccl_comm_destroy": (None, [c_void_p]),
@@ -98,7 +100,8 @@ def lib():
 EXPORTED = [
     "sdag_plan_opts_init", "sdag_plan_create", "sdag_plan_info_get", "sdag_plan_arg", "sdag_plan_variant_name",
     "sdag_plan_describe", "sdag_plan_destroy", "sdag_apply", "sdag_apply_batched", "sdag_apply_iterated",
-    "sdag_apply_host", "sdag_fusion_schedule", "sdag_slab_partition", "sdag_slab_halo", "sdag_nccl_get_unique_id", "sdag_nccl_comm_create",
+    "sdag_apply_host", "sdag_fusion_schedule", "sdag_slab_partition", "sdag_slab_halo",
+    "sdag_slab_partition2", "sdag_slab_halo2", "sdag_nccl_get_unique_id", "sdag_nccl_comm_create",
     "sdag_nccl_comm_destroy", "sdag_dist_create", "sdag_dist_layout", "sdag_dist_local_plan", "sdag_dist_apply",
     "sdag_dist_apply_iterated", "sdag_dist_destroy", "sdag_dist_apply_iterated_loopback", "sdag_last_error",
     "sdag_version", "sdag_launch_count", "sdag_measure_fp64_peak", "sdag_registry_count", "sdag_registry_get",

@@ -49,6 +49,7 @@ void sdag_plan_opts_init(sdag_plan_opts *o) {
     o->batch = 1;
     o->force_variant = nullptr;
     o->fusion = 1;
+    o->time_tile = 1;
 }
 
 sdag_status sdag_plan_create(const char *spec, const int64_t dims[3], const sdag_plan_opts *opts, sdag_plan *out) {
@@ -172,6 +173,35 @@ sdag_status sdag_slab_halo(int64_t global_nz, int32_t rz, int32_t nranks, int32_
     });
 }
 
+sdag_status sdag_slab_partition2(int64_t global_nz, int32_t rz, int32_t time_tile, int32_t nranks, int32_t rank,
+                                 int64_t out[8]) {
+    return guard([&] {
+        if (!out) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null out");
+        sdag::Slab s = sdag::slab_partition(global_nz, rz, nranks, rank, time_tile);
+        out[0] = s.z0;
+        out[1] = s.nz_own;
+        out[2] = s.nz_alloc;
+        out[3] = s.k_lo;
+        out[4] = s.k_hi;
+        out[5] = s.has_lower;
+        out[6] = s.has_upper;
+        out[7] = s.halo;
+    });
+}
+
+sdag_status sdag_slab_halo2(int64_t global_nz, int32_t rz, int32_t time_tile, int32_t nranks, int32_t rank,
+                            int32_t planes, int64_t out[5]) {
+    return guard([&] {
+        if (!out) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null out");
+        sdag::Halo h = sdag::halo_schedule(sdag::slab_partition(global_nz, rz, nranks, rank, time_tile), planes);
+        out[0] = h.lo_send;
+        out[1] = h.lo_recv;
+        out[2] = h.up_send;
+        out[3] = h.up_recv;
+        out[4] = h.planes;
+    });
+}
+
 sdag_status sdag_nccl_get_unique_id(uint8_t id[128]) {
     return guard([&] { sdag::nccl_unique_id(id); });
 }
@@ -198,7 +228,7 @@ sdag_status sdag_dist_layout(sdag_dist d, int64_t local_dims[3], int64_t *gz0) {
         auto *D = reinterpret_cast<sdag::Dist *>(d);
         if (!D) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null dist");
         for (int a = 0; a < 3; a++) local_dims[a] = D->local->dims[a];
-        if (gz0) *gz0 = D->slab.z0 - D->rz;
+        if (gz0) *gz0 = D->slab.z0 - D->slab.halo;
     });
 }
 

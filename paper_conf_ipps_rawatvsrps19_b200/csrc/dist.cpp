@@ -25,20 +25,23 @@ namespace sdag {
 // host logic
 // ---------------------------------------------------------------------------
 
-Slab slab_partition(int64_t gnz, int rz, int nranks, int rank) {
+Slab slab_partition(int64_t gnz, int rz, int nranks, int rank, int time_tile) {
     if (nranks < 1 || rank < 0 || rank >= nranks) throw Error(SDAG_ERR_INVALID_ARG, "bad rank / nranks");
     if (rz < 0) throw Error(SDAG_ERR_INVALID_ARG, "negative radius");
+    if (time_tile < 1 || time_tile > 7) throw Error(SDAG_ERR_INVALID_ARG, "time_tile must be in 1..7");
+    const int64_t H = int64_t(rz) * time_tile;
     if (gnz < 2 * int64_t(rz) + 1) throw Error(SDAG_ERR_DOMAIN, "global z extent has no interior");
     Slab s;
     const int64_t base = gnz / nranks, rem = gnz % nranks;
     s.nz_own = base + (rank < rem ? 1 : 0);
     s.z0 = int64_t(rank) * base + std::min<int64_t>(rank, rem);
-    if (base < std::max(rz, 1))
-        throw Error(SDAG_ERR_DOMAIN, "every rank must own at least max(R_z,1) = " + std::to_string(std::max(rz, 1)) +
-                                         " planes (global nz " + std::to_string(gnz) + ", " +
-                                         std::to_string(nranks) + " ranks)");
-    s.nz_alloc = s.nz_own + 2 * rz;
-    const int64_t g_of_l0 = s.z0 - rz;  // global plane of local plane 0
+    if (base < std::max<int64_t>(H, 1))
+        throw Error(SDAG_ERR_DOMAIN, "every rank must own at least max(R_z*time_tile,1) = " +
+                                         std::to_string(std::max<int64_t>(H, 1)) + " planes (global nz " +
+                                         std::to_string(gnz) + ", " + std::to_string(nranks) + " ranks)");
+    s.halo = H;
+    s.nz_alloc = s.nz_own + 2 * H;
+    const int64_t g_of_l0 = s.z0 - H;  // global plane of local plane 0
     const int64_t glo = std::max<int64_t>(s.z0, rz), ghi = std::min<int64_t>(s.z0 + s.nz_own, gnz - rz);
     s.k_lo = glo - g_of_l0;
     s.k_hi = std::max(ghi - g_of_l0, s.k_lo);
@@ -47,17 +50,19 @@ Slab slab_partition(int64_t gnz, int rz, int nranks, int rank) {
     return s;
 }
 
-Halo halo_schedule(const Slab &s, int rz) {
+Halo halo_schedule(const Slab &s, int planes) {
     Halo h;
-    h.planes = rz;
-    if (rz == 0) return h;
+    if (planes < 0 || planes > s.halo) throw Error(SDAG_ERR_INVALID_ARG, "halo planes must be in 0..H");
+    h.planes = planes;
+    if (planes == 0) return h;
+    const int64_t H = s.halo;
     if (s.has_lower) {
-        h.lo_send = rz;  // my lowest rz owned planes
-        h.lo_recv = 0;   // ghosts below
+        h.lo_send = H;           // my lowest `planes` owned planes
+        h.lo_recv = H - planes;  // the ghosts right below them
     }
     if (s.has_upper) {
-        h.up_send = s.nz_alloc - 2 * rz;  // my highest rz owned planes
-        h.up_recv = s.nz_alloc - rz;      // ghosts above
+        h.up_send = H + s.nz_own - planes;  // my highest `planes` owned planes
+        h.up_recv = H + s.nz_own;           // the ghosts right above them
     }
     return h;
 }
@@ -161,9 +166,6 @@ Dist::~Dist() {
 
 Dist *dist_create(const std::string &spec, const int64_t gdims[3], const sdag_plan_opts &o, int rank, int nranks,
                   void *comm) {
-    if (nranks > 1 && !comm && o.device != SDAG_DEVICE_NONE) {
-        // allowed: loopback use (dist_apply_iterated_loopback); NCCL entry points check comm
-    }
     // analyse once on the global grid to get R_z (host-only)
     sdag_plan_opts ho = o;
     ho.device = SDAG_DEVICE_NONE;
@@ -171,8 +173,10 @@ Dist *dist_create(const std::string &spec, const int64_t gdims[3], const sdag_pl
     std::unique_ptr<Plan> g(plan_create(spec, gdims, ho));
     const int rz = g->an.radius[0];
     std::unique_ptr<Dist> d(new Dist());
-    d->slab = slab_partition(gdims[0], rz, nranks, rank);
+    d->time_tile = std::max(1, int(o.time_tile));
+    d->slab = slab_partition(gdims[0], rz, nranks, rank, d->time_tile);
     d->rz = rz;
+    d->gnz = gdims[0];
     d->rank = rank;
     d->nranks = nranks;
     d->comm = comm;
@@ -194,25 +198,31 @@ struct Ranges {
     int64_t b_lo[2] = {0, 0}, b_hi[2] = {0, 0};  // lower / upper boundary bands
 };
 
-Ranges ranges_of(const Dist *d) {
+// Output planes of one launch whose inputs reach `depth` planes in z (R_z for
+// a sweep, x R_z for an x-sweep fused launch): the interior range reads no
+// ghost plane and can overlap the exchange; the two bands next to the ghost
+// layers run after it.
+Ranges ranges_of(const Dist *d, int64_t depth) {
     const Slab &s = d->slab;
-    const int64_t rz = d->rz;
+    const int64_t H = s.halo;
     Ranges r;
-    if (rz == 0 || s.nz_own < 2 * rz) {  // nothing to overlap: one launch after the exchange
+    if (depth == 0 || s.nz_own < 2 * depth) {  // nothing to overlap: one launch after the exchange
         r.split = false;
         r.b_lo[0] = s.k_lo;
         r.b_hi[0] = s.k_hi;
         return r;
     }
-    r.in_lo = s.has_lower ? 2 * rz : s.k_lo;
-    r.in_hi = s.has_upper ? s.nz_alloc - 2 * rz : s.k_hi;
+    r.in_lo = s.has_lower ? H + depth : s.k_lo;
+    r.in_hi = s.has_upper ? H + s.nz_own - depth : s.k_hi;
+    r.in_lo = std::max(r.in_lo, s.k_lo);
+    r.in_hi = std::min(r.in_hi, s.k_hi);
     if (s.has_lower) {
-        r.b_lo[0] = std::max<int64_t>(rz, s.k_lo);
-        r.b_hi[0] = std::min<int64_t>(2 * rz, s.k_hi);
+        r.b_lo[0] = std::max<int64_t>(H, s.k_lo);
+        r.b_hi[0] = std::min<int64_t>(H + depth, s.k_hi);
     }
     if (s.has_upper) {
-        r.b_lo[1] = std::max<int64_t>(s.nz_alloc - 2 * rz, s.k_lo);
-        r.b_hi[1] = std::min<int64_t>(s.nz_alloc - rz, s.k_hi);
+        r.b_lo[1] = std::max<int64_t>(H + s.nz_own - depth, s.k_lo);
+        r.b_hi[1] = std::min<int64_t>(H + s.nz_own, s.k_hi);
     }
     return r;
 }
@@ -228,14 +238,14 @@ std::vector<int> halo_arrays(const Dist *d) {
     return v;
 }
 
-void exchange_nccl(Dist *d, double *const *a3, cudaStream_t comm) {
-    if (d->rz == 0 || d->nranks == 1) return;
+void exchange_nccl(Dist *d, double *const *a3, cudaStream_t comm, int planes) {
+    if (planes == 0 || d->nranks == 1) return;
     if (!d->comm) throw Error(SDAG_ERR_INVALID_ARG, "multi-rank dist without an NCCL communicator");
     const NcclApi &N = nccl();
     const Plan *p = d->local;
     const size_t plane = size_t(p->dims[1] * p->dims[2]);
-    const size_t cnt = plane * size_t(d->rz);
-    const Halo h = halo_schedule(d->slab, d->rz);
+    const size_t cnt = plane * size_t(planes);
+    const Halo h = halo_schedule(d->slab, planes);
     auto c = static_cast<ncclComm_t>(d->comm);
     nck(N.GroupStart(), "ncclGroupStart");
     for (int f : halo_arrays(d)) {
@@ -252,28 +262,75 @@ void exchange_nccl(Dist *d, double *const *a3, cudaStream_t comm) {
     nck(N.GroupEnd(), "ncclGroupEnd");
 }
 
-void sweep_split(Dist *d, double *const *a3, const double *const *a1, const double *s, cudaStream_t compute,
-                 cudaStream_t comm, bool do_exchange) {
+// local planes of the global z-interior (multi-sweep kernels keep the rest fixed)
+void global_interior(const Dist *d, int64_t zr[2]) {
+    const Slab &s = d->slab;
+    const int64_t g_of_l0 = s.z0 - s.halo;
+    const int64_t gnz = d->gnz;
+    zr[0] = d->rz - g_of_l0;
+    zr[1] = gnz - d->rz - g_of_l0;
+}
+
+// One launch of kernel `k` (x = k.tsteps sweeps) with its exchange of x R_z planes.
+void sweep_split(Dist *d, const KernelDesc &k, double *const *a3, const double *const *a1, const double *s,
+                 cudaStream_t compute, cudaStream_t comm, bool do_exchange) {
     Plan *p = d->local;
-    const KernelDesc &k = p->kernel();
-    const Ranges r = ranges_of(d);
-    const bool xchg = do_exchange && d->rz > 0 && d->nranks > 1;
+    const int64_t depth = int64_t(d->rz) * k.tsteps;
+    const Ranges r = ranges_of(d, depth);
+    const bool xchg = do_exchange && depth > 0 && d->nranks > 1;
+    int64_t zr[2];
+    global_interior(d, zr);
     if (xchg) {
         check_cuda(cudaEventRecord(d->ev_ready, compute), "cudaEventRecord");
         check_cuda(cudaStreamWaitEvent(comm, d->ev_ready, 0), "cudaStreamWaitEvent");
-        exchange_nccl(d, a3, comm);
+        exchange_nccl(d, a3, comm, int(depth));
         check_cuda(cudaEventRecord(d->ev_halo, comm), "cudaEventRecord");
     }
-    if (r.split && r.in_hi > r.in_lo) plan_launch(p, k, const_cast<double *const *>(a3), a1, s, 1, r.in_lo, r.in_hi, compute);
+    double *const *a = const_cast<double *const *>(a3);
+    if (r.split && r.in_hi > r.in_lo) plan_launch(p, k, a, a1, s, 1, r.in_lo, r.in_hi, compute, nullptr, zr);
     if (xchg) check_cuda(cudaStreamWaitEvent(compute, d->ev_halo, 0), "cudaStreamWaitEvent");
     for (int q = 0; q < 2; q++)
-        if (r.b_hi[q] > r.b_lo[q]) plan_launch(p, k, const_cast<double *const *>(a3), a1, s, 1, r.b_lo[q], r.b_hi[q], compute);
+        if (r.b_hi[q] > r.b_lo[q]) plan_launch(p, k, a, a1, s, 1, r.b_lo[q], r.b_hi[q], compute, nullptr, zr);
 }
 
 cudaStream_t comm_stream(Dist *d, cudaStream_t comm) {
     if (comm) return comm;
     if (!d->own_comm) check_cuda(cudaStreamCreateWithFlags(&d->own_comm, cudaStreamNonBlocking), "cudaStreamCreate");
     return d->own_comm;
+}
+
+// the launch schedule of T sweeps on this slab: fused kernels of up to
+// time_tile sweeps (their exchange depth fits the ghost layer), deep-tuning DP
+std::vector<const KernelDesc *> iter_schedule(Dist *d, double *b0, double *b1, int T) {
+    Plan *p = d->local;
+    const KernelDesc *fk[8] = {nullptr};
+    int maxdeg = 1;
+    const bool aligned = (reinterpret_cast<uintptr_t>(b0) % 16) == 0 && (reinterpret_cast<uintptr_t>(b1) % 16) == 0;
+    if (p->fusion && aligned && p->dims[2] % 2 == 0)
+        for (const KernelDesc *f : p->fused)
+            if (f->tsteps <= d->time_tile && !fk[f->tsteps]) {
+                fk[f->tsteps] = f;
+                maxdeg = std::max(maxdeg, f->tsteps);
+            }
+    double f[8];
+    for (int x = 0; x < 8; x++) f[x] = (x == 1 || (x > 1 && x <= maxdeg && fk[x])) ? p->fcost[x] : 0.0;
+    std::vector<const KernelDesc *> seq;
+    for (int x : fusion_schedule(f, maxdeg, T)) {
+        if (x == 1) {
+            seq.push_back(nullptr);  // the plan's single-sweep kernel (picked per launch for alignment)
+        } else {
+            seq.push_back(fk[x]);
+        }
+    }
+    return seq;
+}
+
+const KernelDesc &single_kernel(Plan *p, double *in) {
+    const KernelDesc &k = p->kernel();
+    if (!k.tma || (reinterpret_cast<uintptr_t>(in) % 16 == 0 && p->dims[2] % 2 == 0)) return k;
+    for (const KernelDesc *c : p->cands)
+        if (!c->tma && c->tx == k.tx && c->ty == k.ty && c->ux == k.ux && c->uy == k.uy && c->pf == k.pf) return *c;
+    throw Error(SDAG_ERR_INVALID_ARG, "arrays are not 16-byte aligned and no LSU variant exists");
 }
 
 }  // namespace
@@ -290,7 +347,7 @@ void dist_apply(Dist *d, double *const *a3, int n3, const double *const *a1, int
         for (int f = 0; f < n3; f++)
             if (reinterpret_cast<uintptr_t>(a3[f]) % 16) throw Error(SDAG_ERR_INVALID_ARG, "grid arrays must be 16-B aligned");
     check_cuda(cudaSetDevice(p->device), "cudaSetDevice");  // libsdag's runtime: bind the plan's device
-    sweep_split(d, a3, a1, s, compute, comm_stream(d, comm), true);
+    sweep_split(d, p->kernel(), a3, a1, s, compute, comm_stream(d, comm), true);
 }
 
 void dist_apply_iterated(Dist *d, double *b0, double *b1, int T, const double *s, int ns, cudaStream_t compute,
@@ -300,17 +357,19 @@ void dist_apply_iterated(Dist *d, double *b0, double *b1, int T, const double *s
     if (p->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
     if (p->n3() != 2 || p->an.n_in != 1 || p->an.n_out != 1 || p->n1() != 0)
         throw Error(SDAG_ERR_INVALID_ARG, "iterated dist apply needs a 1-input 1-output plan");
-    if (ns != p->ns() || !b0 || !b1 || b0 == b1) throw Error(SDAG_ERR_INVALID_ARG, "bad arguments");
+    if (ns != p->ns() || !b0 || !b1 || b0 == b1 || T < 0) throw Error(SDAG_ERR_INVALID_ARG, "bad arguments");
     int fin = -1, fout = -1;
     for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
     check_cuda(cudaSetDevice(p->device), "cudaSetDevice");
     cudaStream_t cs = comm_stream(d, comm);
     double *bufs[2] = {b0, b1};
-    for (int t = 0; t < T; t++) {
+    int cur = 0;
+    for (const KernelDesc *k : iter_schedule(d, b0, b1, T)) {
         double *a3[2];
-        a3[fin] = bufs[t & 1];
-        a3[fout] = bufs[(t + 1) & 1];
-        sweep_split(d, a3, nullptr, s, compute, cs, true);
+        a3[fin] = bufs[cur];
+        a3[fout] = bufs[1 - cur];
+        sweep_split(d, k ? *k : single_kernel(p, bufs[cur]), a3, nullptr, s, compute, cs, true);
+        cur = 1 - cur;
     }
 }
 
@@ -320,31 +379,37 @@ void dist_apply_iterated_loopback(Dist **ds, int n, double *const *b0, double *c
     for (int r = 0; r < n; r++) {
         if (!ds[r] || ds[r]->rank != r || ds[r]->nranks != n) throw Error(SDAG_ERR_INVALID_ARG, "dists must be ranks 0..n-1");
         if (ds[r]->local->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
+        if (ds[r]->time_tile != ds[0]->time_tile) throw Error(SDAG_ERR_INVALID_ARG, "dists must share time_tile");
     }
     Plan *p0 = ds[0]->local;
-    if (p0->n3() != 2 || p0->an.n_in != 1 || p0->an.n_out != 1 || p0->n1() != 0 || ns != p0->ns())
+    if (p0->n3() != 2 || p0->an.n_in != 1 || p0->an.n_out != 1 || p0->n1() != 0 || ns != p0->ns() || T < 0)
         throw Error(SDAG_ERR_INVALID_ARG, "iterated loopback needs a 1-input 1-output plan");
     int fin = -1, fout = -1;
     for (int f = 0; f < 2; f++) (p0->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
     check_cuda(cudaSetDevice(p0->device), "cudaSetDevice");
     const int64_t rz = ds[0]->rz;
     const size_t plane = size_t(p0->dims[1] * p0->dims[2]);
-    for (int t = 0; t < T; t++) {
+    // every rank follows rank 0's schedule (same plan, same buffers' alignment class)
+    const std::vector<const KernelDesc *> sched = iter_schedule(ds[0], b0[0], b1[0], T);
+    int t = 0;
+    for (const KernelDesc *k0 : sched) {
         auto in = [&](int r) { return (t & 1) ? b1[r] : b0[r]; };
         auto out = [&](int r) { return (t & 1) ? b0[r] : b1[r]; };
-        if (rz > 0) {
+        const int x = k0 ? k0->tsteps : 1;
+        const int planes = int(rz) * x;
+        if (planes > 0) {
             for (int r = 0; r < n; r++) {  // the same schedule the NCCL path sends/receives
-                const Halo h = halo_schedule(ds[r]->slab, int(rz));
+                const Halo h = halo_schedule(ds[r]->slab, planes);
                 if (h.lo_recv >= 0) {  // from the lower neighbour's upper send band
-                    const Halo hl = halo_schedule(ds[r - 1]->slab, int(rz));
+                    const Halo hl = halo_schedule(ds[r - 1]->slab, planes);
                     check_cuda(cudaMemcpyAsync(in(r) + size_t(h.lo_recv) * plane, in(r - 1) + size_t(hl.up_send) * plane,
-                                               size_t(rz) * plane * 8, cudaMemcpyDeviceToDevice, stream),
+                                               size_t(planes) * plane * 8, cudaMemcpyDeviceToDevice, stream),
                                "loopback halo");
                 }
                 if (h.up_recv >= 0) {  // from the upper neighbour's lower send band
-                    const Halo hu = halo_schedule(ds[r + 1]->slab, int(rz));
+                    const Halo hu = halo_schedule(ds[r + 1]->slab, planes);
                     check_cuda(cudaMemcpyAsync(in(r) + size_t(h.up_recv) * plane, in(r + 1) + size_t(hu.lo_send) * plane,
-                                               size_t(rz) * plane * 8, cudaMemcpyDeviceToDevice, stream),
+                                               size_t(planes) * plane * 8, cudaMemcpyDeviceToDevice, stream),
                                "loopback halo");
                 }
             }
@@ -353,8 +418,9 @@ void dist_apply_iterated_loopback(Dist **ds, int n, double *const *b0, double *c
             double *a3[2];
             a3[fin] = in(r);
             a3[fout] = out(r);
-            sweep_split(ds[r], a3, nullptr, s, stream, stream, false);
+            sweep_split(ds[r], k0 ? *k0 : single_kernel(ds[r]->local, in(r)), a3, nullptr, s, stream, stream, false);
         }
+        t++;
     }
 }
 

@@ -12,25 +12,31 @@ namespace sdag {
 struct Slab {
     int64_t z0 = 0;        // first owned global plane
     int64_t nz_own = 0;    // owned planes
-    int64_t nz_alloc = 0;  // owned + 2 rz (ghosts below and above)
+    int64_t halo = 0;      // ghost planes per side H = R_z x time tile
+    int64_t nz_alloc = 0;  // owned + 2 H (ghosts below and above)
     int64_t k_lo = 0, k_hi = 0;  // local planes computed (global interior only)
     int has_lower = 0, has_upper = 0;
 };
-Slab slab_partition(int64_t global_nz, int rz, int nranks, int rank);
+// time_tile t >= 1: ghost depth H = R_z t, so t sweeps can run between
+// exchanges (communication-avoiding temporal fusion).
+Slab slab_partition(int64_t global_nz, int rz, int nranks, int rank, int time_tile = 1);
 
-// Halo schedule of one sweep, in LOCAL plane indices, rz planes each:
-// to the lower neighbour send [lo_send, lo_send+rz) and receive into
-// [lo_recv, lo_recv+rz); likewise for the upper neighbour.  -1 = no neighbour.
+// Halo schedule of one exchange of `planes` (<= H) planes per side, in LOCAL
+// plane indices: to the lower neighbour send [lo_send, lo_send+planes) and
+// receive into [lo_recv, lo_recv+planes); likewise for the upper neighbour.
+// -1 = no neighbour.
 struct Halo {
     int64_t lo_send = -1, lo_recv = -1, up_send = -1, up_recv = -1, planes = 0;
 };
-Halo halo_schedule(const Slab &s, int rz);
+Halo halo_schedule(const Slab &s, int planes);
 
 struct Dist {
     Plan *local = nullptr;  // plan over the local allocation (nz_alloc, ny, nx)
     sdag_plan_s handle{nullptr};
     Slab slab;
     int rz = 0;
+    int time_tile = 1;      // sweeps a fused launch may take between exchanges (H = rz * time_tile)
+    int64_t gnz = 0;        // global z extent
     int rank = 0, nranks = 1;
     void *comm = nullptr;   // ncclComm_t (not owned)
     cudaStream_t own_comm = nullptr;

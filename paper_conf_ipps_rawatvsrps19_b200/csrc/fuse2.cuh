@@ -61,7 +61,7 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX>::THREADS, MINB)
     if (kb >= ke) return;
     const int p0 = kb - 2, plast = ke + 1;  // input planes streamed
     const int64_t zbase = prob * a.nz;
-    const int nz = int(a.nz), ny = int(a.ny), nx = int(a.nx);
+    const int ny = int(a.ny), nx = int(a.nx);
 
     const int t = threadIdx.x;
     const int lx = t % G::NTX, ly = t / G::NTX;
@@ -151,7 +151,7 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX>::THREADS, MINB)
             asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[unsigned(p - p0) % NS]))
                          : "memory");
         const int j = p - 1;
-        const bool zring = j <= 0 || j >= nz - 1;
+        const bool zring = j < a.zr_lo || j >= a.zr_hi;
         double *s1 = s1buf + (j & 1) * PAL;
 #pragma unroll
         for (int py = 0; py < UY; py++) {

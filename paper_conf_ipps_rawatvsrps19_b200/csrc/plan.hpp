@@ -72,7 +72,7 @@ void plan_fill_info(Plan *p, sdag_plan_info *info);
 // interior); all arrays are per-problem [batch][nz][ny][nx].
 void plan_launch(Plan *p, const KernelDesc &k, double *const *arrays3d, const double *const *arrays1d,
                  const double *scalars, int batch, int64_t klo, int64_t khi, cudaStream_t stream,
-                 const int64_t *dims_override = nullptr);
+                 const int64_t *dims_override = nullptr, const int64_t *zr = nullptr);
 void apply(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns, int batch,
            cudaStream_t stream);
 std::vector<int> fusion_schedule(const double *f, int maxdeg, int T);

@@ -179,7 +179,7 @@ static const KernelDesc &pick_kernel(Plan *p, double *const *a3, int64_t nx) {
 }
 
 void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *const *a1, const double *s, int batch,
-                 int64_t klo, int64_t khi, cudaStream_t stream, const int64_t *dims_override) {
+                 int64_t klo, int64_t khi, cudaStream_t stream, const int64_t *dims_override, const int64_t *zr) {
     const int64_t *dims = dims_override ? dims_override : p->dims;
     int64_t lo[3], hi[3];
     for (int a = 0; a < 3; a++) {
@@ -214,6 +214,11 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *
     A.nx = dims[2];
     A.ny = dims[1];
     A.nz = dims[0];
+    // planes a multi-sweep kernel may update (its intermediate sweeps keep the
+    // global z-ring fixed, reading R1); a z-slab passes its global ring's
+    // local position
+    A.zr_lo = int32_t(zr ? zr[0] : lo[0]);
+    A.zr_hi = int32_t(zr ? zr[1] : hi[0]);
     A.lo[0] = int32_t(klo);
     A.hi[0] = int32_t(khi);
     for (int a = 1; a < 3; a++) {

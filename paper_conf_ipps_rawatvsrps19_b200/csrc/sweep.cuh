@@ -66,6 +66,7 @@ struct SweepArgs {
     int32_t lo[3], hi[3];         // output point range per axis (z, y, x)
     int32_t tiles_x, tiles_y, nchunk, zchunk;
     int32_t xmin;                 // first interior x (lo[2] may be rounded down to even as tile origin)
+    int32_t zr_lo, zr_hi;         // multi-sweep kernels: planes [zr_lo, zr_hi) are global interior (others ring)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {

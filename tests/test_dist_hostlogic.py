@@ -48,6 +48,31 @@ def test_halo_schedule_pairs_up():
     assert sdag.slab_halo(gnz, rz, P, P - 1)["up_send"] == -1
 
 
+@pytest.mark.parametrize("gnz,rz,tt,P", [(40, 1, 2, 2), (41, 1, 3, 4), (50, 2, 2, 3), (64, 4, 2, 4)])
+def test_time_tiled_partition_and_halo(gnz, rz, tt, P):
+    """Ghost depth H = R_z t; the same owned planes as t = 1; exchanges of any
+    planes <= H pair up between neighbours on the same global planes."""
+    H = rz * tt
+    for r in range(P):
+        a = sdag.slab_partition(gnz, rz, P, r)
+        b = sdag.slab_partition2(gnz, rz, tt, P, r)
+        assert (b["z0"], b["nz_own"], b["halo"]) == (a["z0"], a["nz_own"], H)
+        assert b["nz_alloc"] == b["nz_own"] + 2 * H
+        g0 = b["z0"] - H
+        assert (b["k_lo"] + g0, b["k_hi"] + g0) == (a["k_lo"] + a["z0"] - rz, a["k_hi"] + a["z0"] - rz)
+    for planes in range(1, H + 1):
+        for r in range(P - 1):
+            x = sdag.slab_halo2(gnz, rz, tt, P, r, planes)
+            y = sdag.slab_halo2(gnz, rz, tt, P, r + 1, planes)
+            gx = sdag.slab_partition2(gnz, rz, tt, P, r)["z0"] - H
+            gy = sdag.slab_partition2(gnz, rz, tt, P, r + 1)["z0"] - H
+            assert gx + x["up_send"] == gy + y["lo_recv"] and gy + y["lo_send"] == gx + x["up_recv"]
+            # the received planes sit right next to the owned range
+            assert y["lo_recv"] + planes == H and x["up_recv"] == H + sdag.slab_partition2(gnz, rz, tt, P, r)["nz_own"]
+    with pytest.raises(sdag.SdagError):
+        sdag.slab_halo2(gnz, rz, tt, P, 0, H + 1)
+
+
 def test_partition_errors():
     with pytest.raises(sdag.SdagError) as e:
         sdag.slab_partition(20, 4, 8, 0)  # 2 planes per rank < R_z
@@ -64,7 +89,11 @@ def _free_port():
     return p
 
 
-def _worker(rank, P, port, gdims, T, q):
+def _worker(rank, P, port, gdims, T, q, tt=1):
+    """One rank: its slab + ghosts; per launch of x sweeps (x <= time tile tt,
+    the apply_iterated DP schedule) ONE exchange of x*R_z planes, then x oracle
+    sweeps, the i-th on the owned range widened by (x-i)*R_z planes into the
+    ghosts (the redundant computation of communication-avoiding fusion)."""
     import torch
     import torch.distributed as dist
 
@@ -77,44 +106,57 @@ def _worker(rank, P, port, gdims, T, q):
         rz = 1
         A = synth.uniform(gdims, -1, 1, "gloo-slab")  # each rank regenerates the same global field
         w, nu = [-128 / 30, 14 / 30, 3 / 30, 1 / 30], 0.125
-        s = sd.slab_partition(gdims[0], rz, P, rank)
-        h = sd.slab_halo(gdims[0], rz, P, rank)
-        g0 = s["z0"] - rz
+        s = sd.slab_partition2(gdims[0], rz, tt, P, rank)
+        H = s["halo"]
+        g0 = s["z0"] - H
+        zr_lo, zr_hi = rz - g0, gdims[0] - rz - g0  # local planes of the global interior
         loc = np.zeros((s["nz_alloc"], *gdims[1:]))
         lo, hi = max(g0, 0), min(g0 + s["nz_alloc"], gdims[0])
         loc[lo - g0:hi - g0] = A[lo:hi]
         bufs = [loc, loc.copy()]
-        for t in range(T):
-            src, dst = bufs[t & 1], bufs[(t + 1) & 1]
+        sched = sd.fusion_schedule({1: 1.0, **({tt: 1.0 + 0.15 * (tt - 1)} if tt > 1 else {})}, T)[0]
+        t = 0
+        for x in sched:
+            src = bufs[t & 1]
+            h = sd.slab_halo2(gdims[0], rz, tt, P, rank, x * rz)
+            n = h["planes"]
             reqs = []
             if h["lo_send"] >= 0:
-                reqs.append(dist.isend(torch.from_numpy(src[h["lo_send"]:h["lo_send"] + rz].copy()), rank - 1))
-                rb = torch.empty((rz, *gdims[1:]), dtype=torch.float64)
+                reqs.append(dist.isend(torch.from_numpy(src[h["lo_send"]:h["lo_send"] + n].copy()), rank - 1))
+                rb = torch.empty((n, *gdims[1:]), dtype=torch.float64)
                 reqs.append(("recv", dist.irecv(rb, rank - 1), rb, h["lo_recv"]))
             if h["up_send"] >= 0:
-                reqs.append(dist.isend(torch.from_numpy(src[h["up_send"]:h["up_send"] + rz].copy()), rank + 1))
-                rb2 = torch.empty((rz, *gdims[1:]), dtype=torch.float64)
+                reqs.append(dist.isend(torch.from_numpy(src[h["up_send"]:h["up_send"] + n].copy()), rank + 1))
+                rb2 = torch.empty((n, *gdims[1:]), dtype=torch.float64)
                 reqs.append(("recv", dist.irecv(rb2, rank + 1), rb2, h["up_recv"]))
             for r_ in reqs:
                 if isinstance(r_, tuple):
                     r_[1].wait()
-                    src[r_[3]:r_[3] + rz] = r_[2].numpy()
+                    src[r_[3]:r_[3] + n] = r_[2].numpy()
                 else:
                     r_.wait()
-            oracle.smooth27(src, w, nu, out=dst, krange=(s["k_lo"], s["k_hi"]))
+            for i in range(1, x + 1):
+                src, dst = bufs[t & 1], bufs[(t + 1) & 1]
+                ext = (x - i) * rz
+                klo = max(s["k_lo"] - (ext if s["has_lower"] else 0), zr_lo)
+                khi = min(s["k_hi"] + (ext if s["has_upper"] else 0), zr_hi)
+                oracle.smooth27(src, w, nu, out=dst, krange=(klo, khi))
+                t += 1
         res = bufs[T & 1][s["z0"] - g0:s["z0"] - g0 + s["nz_own"]]
         q.put((rank, s["z0"], res))
     finally:
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("P", [2, 3])
-def test_gloo_slab_iteration_equals_global_oracle(P):
-    gdims, T = (17, 9, 10), 4
+@pytest.mark.parametrize("P,tt,T", [(2, 1, 4), (3, 1, 4), (2, 2, 5), (3, 2, 6)])
+def test_gloo_slab_iteration_equals_global_oracle(P, tt, T):
+    """tt = 2: communication-avoiding temporal fusion (NEXT-1) -- one exchange of
+    2 R_z planes per fused pair of sweeps -- still equals the global iteration."""
+    gdims = (17, 9, 10)
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, P, port, gdims, T, q)) for r in range(P)]
+    procs = [ctx.Process(target=_worker, args=(r, P, port, gdims, T, q, tt)) for r in range(P)]
     for p in procs:
         p.start()
     parts = [q.get(timeout=180) for _ in range(P)]

@@ -187,11 +187,15 @@ def test_apply_host_end_to_end():
     check("lap25", dims, [out], case)
 
 
-@pytest.mark.parametrize("name,gdims,T", [("smooth27", (30, 20, 22), 6), ("lap25", (44, 18, 20), 3)])
+@pytest.mark.parametrize("name,gdims,T,tt", [("smooth27", (30, 20, 22), 6, 1), ("lap25", (44, 18, 20), 3, 1),
+                                             ("smooth27", (30, 20, 22), 6, 2), ("smooth27", (31, 22, 24), 5, 2),
+                                             ("smooth27", (40, 26, 30), 12, 2)])
 @pytest.mark.parametrize("P", [1, 2, 3, 4])
-def test_loopback_slabs_bitwise_equal_single_gpu(name, gdims, T, P):
+def test_loopback_slabs_bitwise_equal_single_gpu(name, gdims, T, tt, P):
     """a7 bookkeeping: P z-slabs with the halo schedule of the NCCL path
-    (moved by cudaMemcpy) reproduce the single-GPU iteration bit for bit."""
+    (moved by cudaMemcpy) reproduce the single-GPU iteration bit for bit.
+    tt = 2 (NEXT-1, communication-avoiding): ghost depth 2 R_z, fused 2-sweep
+    launches, one exchange of 2 R_z planes per launch."""
     case = make_case(name, gdims, cfg="slab")
     A = case["inputs"][0]
     s = case["s"]
@@ -202,7 +206,7 @@ def test_loopback_slabs_bitwise_equal_single_gpu(name, gdims, T, P):
     full.apply_iterated(b0, b1, T, scalars=s)
     ref = (b0 if T % 2 == 0 else b1).cpu().numpy()
 
-    dists = [sdag.Dist(spec, gdims, r, P) for r in range(P)]
+    dists = [sdag.Dist(spec, gdims, r, P, time_tile=tt) for r in range(P)]
     bufs0, bufs1 = [], []
     for d in dists:
         (nza, ny, nx), g0 = d.layout()
@@ -211,11 +215,15 @@ def test_loopback_slabs_bitwise_equal_single_gpu(name, gdims, T, P):
         loc[lo - g0:hi - g0] = A[lo:hi]
         bufs0.append(torch.from_numpy(loc).cuda())
         bufs1.append(torch.from_numpy(loc.copy()).cuda())
+    n0 = sdag.launch_count()
     sdag.Dist.apply_iterated_loopback(dists, bufs0, bufs1, T, scalars=s)
     torch.cuda.synchronize()
+    nl = sdag.launch_count() - n0
+    if tt == 2 and T >= 4:  # fused launches: at most 3 per rank per pair of sweeps
+        assert nl <= P * 3 * ((T + 1) // 2 + 1) and nl < P * 3 * T
     res = bufs0 if T % 2 == 0 else bufs1
     for r, d in enumerate(dists):
-        part = sdag.slab_partition(gdims[0], RADIUS[name], P, r)
+        part = sdag.slab_partition2(gdims[0], RADIUS[name], tt, P, r)
         (nza, ny, nx), g0 = d.layout()
         z0, n = part["z0"], part["nz_own"]
         got = res[r].cpu().numpy()[z0 - g0:z0 - g0 + n]

@@ -1,0 +1,3 @@
+cd $GRAFT_REPO_ROOT
+timeout 900 python tools/perf_sweep.py rhs4center --only tma > gpurun_out/perf_rhs4.jsonl 2> gpurun_out/perf_rhs4.err
+timeout 600 python -m pytest tests/test_gpu_parity.py -q -m gpu --timeout 600 -k "every_variant" > gpurun_out/pytest_var.log 2>&1; echo "exit $?" >> gpurun_out/pytest_var.log
