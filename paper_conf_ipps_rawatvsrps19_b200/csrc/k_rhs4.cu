@@ -4,6 +4,12 @@
 #include "kdesc.cuh"
 namespace sdag {
 void add_kernels_rhs4(std::vector<KernelDesc> &v) {
+    // specialised kernel (rhs4.cuh): 2 x UY patches from 128-bit pair loads, derivative fields
+    // (2 x 2 / 2 x 4 patches spill at 255 registers and run 3x slower; not registered)
+    SDAG_RHS4_PAIR(v, "rhs4center", 32, 16, 1, 1, -10);
+    SDAG_RHS4_PAIR(v, "rhs4center", 16, 16, 1, 1, -9);
+    SDAG_RHS4_PAIR(v, "rhs4center", 64, 8, 1, 1, -8);
+    SDAG_RHS4_PAIR(v, "rhs4center", 32, 8, 1, 1, -7);
     SDAG_PAIR(v, Rhs4, "rhs4center", 16, 16, 1, 1, 1, 0);
     SDAG_PAIR(v, Rhs4, "rhs4center", 32, 8, 1, 1, 1, 1);
     SDAG_PAIR(v, Rhs4, "rhs4center", 16, 16, 1, 2, 1, 2);

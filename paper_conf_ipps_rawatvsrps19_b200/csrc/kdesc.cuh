@@ -9,6 +9,7 @@
 #include "box27.cuh"
 #include "fuse2.cuh"
 #include "hyp.cuh"
+#include "rhs4.cuh"
 #include "star.cuh"
 #include "sweep.cuh"
 
@@ -148,6 +149,42 @@ KernelDesc make_hyp_desc(const char *dag, int prio) {
     do {                                                                          \
         v.push_back(make_hyp_desc<TX, TY, PF, true>(DAG, PRIO));                  \
         v.push_back(make_hyp_desc<TX, TY, PF, false>(DAG, PRIO + 100));           \
+    } while (0)
+
+// rhs4center kernel (rhs4.cuh): 2 x UY patches, derivative fields, 5-plane TMA ring
+template <int TX, int TY, int UY, int PF, bool TMA>
+KernelDesc make_rhs4_desc(const char *dag, int prio) {
+    using G = dev::R4Geo<TX, TY, UY, PF>;
+    KernelDesc d;
+    d.dag = dag;
+    char buf[96];
+    std::snprintf(buf, sizeof buf, "r4_%s_%dx%d_u2x%d_pf%d", TMA ? "tma" : "lsu", TX, TY, UY, PF);
+    d.variant = buf;
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_rhs4<TX, TY, UY, PF, TMA>);
+    d.threads = G::THREADS;
+    d.smem = G::SMEM;
+    d.tx = TX;
+    d.ty = TY;
+    d.ux = 2;
+    d.uy = UY;
+    d.pf = PF;
+    d.tma = TMA;
+    d.nin = 5;
+    d.nout = 3;
+    d.nio = 3;
+    d.n1d = 3;
+    d.rz = 2;
+    d.ry = 2;
+    d.rx = 2;
+    d.rzr = 2;
+    d.prio = prio;
+    return d;
+}
+
+#define SDAG_RHS4_PAIR(v, DAG, TX, TY, UY, PF, PRIO)                               \
+    do {                                                                           \
+        v.push_back(make_rhs4_desc<TX, TY, UY, PF, true>(DAG, PRIO));              \
+        v.push_back(make_rhs4_desc<TX, TY, UY, PF, false>(DAG, PRIO + 100));       \
     } while (0)
 
 // register-capped variant: __launch_bounds__(threads, MINB), TMA only
