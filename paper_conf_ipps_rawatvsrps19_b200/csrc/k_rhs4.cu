@@ -10,6 +10,8 @@ void add_kernels_rhs4(std::vector<KernelDesc> &v) {
     SDAG_RHS4_PAIR(v, "rhs4center", 16, 16, 1, 1, -9);
     SDAG_RHS4_PAIR(v, "rhs4center", 64, 8, 1, 1, -8);
     SDAG_RHS4_PAIR(v, "rhs4center", 32, 8, 1, 1, -7);
+    SDAG_RHS4_PAIR(v, "rhs4center", 32, 16, 1, 2, -6);
+    SDAG_RHS4_PAIR(v, "rhs4center", 16, 32, 1, 1, -5);
     SDAG_PAIR(v, Rhs4, "rhs4center", 16, 16, 1, 1, 1, 0);
     SDAG_PAIR(v, Rhs4, "rhs4center", 32, 8, 1, 1, 1, 1);
     SDAG_PAIR(v, Rhs4, "rhs4center", 16, 16, 1, 2, 1, 2);
