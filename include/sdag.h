@@ -160,10 +160,16 @@ sdag_status sdag_apply_iterated(sdag_plan plan, double *buf0, double *buf1, int3
                                 int32_t nscalars, sdag_stream stream);
 
 /*
- * End-to-end call with HOST buffers (pageable or pinned): copies every 3D
- * input/inout and 1D array host->device into a plan-owned workspace, runs
- * one sweep, copies every output/inout device->host, and synchronises
- * `stream`.  h2d_bytes / d2h_bytes (nullable) receive the bytes moved.
+ * End-to-end call with HOST buffers (pageable or pinned; pinned overlaps):
+ * copies every 3D input/inout and 1D array host->device into a plan-owned
+ * workspace, runs one sweep, copies the interior of every output/inout
+ * device->host (the host ring is not written), and synchronises `stream`.
+ * Pipelined over z-chunks of the output (<= 16 chunks of >= max(8, 2R_z)
+ * planes): the H2D of chunk c+1 (plan-owned copy stream), the sweep of chunk c
+ * (`stream`) and the D2H of chunk c-1 (second copy stream) overlap; every
+ * input plane crosses the link once.  Calls on one plan are serialised.
+ * h2d_bytes / d2h_bytes (nullable) receive the bytes moved.
+ * Errors: INVALID_ARG (counts, null pointers), DEVICE, CUDA, NOMEM.
  */
 sdag_status sdag_apply_host(sdag_plan plan, double *const *host3d, int32_t n3d, const double *const *host1d,
                             int32_t n1d, const double *scalars, int32_t nscalars, sdag_stream stream,

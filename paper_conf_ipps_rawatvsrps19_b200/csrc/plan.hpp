@@ -54,6 +54,9 @@ struct Plan {
     std::map<std::tuple<const void *, int64_t, int64_t, int64_t, int, int>, CUtensorMap> tmaps;
     std::vector<void *> ws;  // sdag_apply_host workspace (device buffers)
     std::vector<size_t> ws_bytes;
+    std::mutex host_mu;              // sdag_apply_host calls on one plan are serialised (shared workspace)
+    cudaStream_t hs_up = nullptr;    // sdag_apply_host copy streams (H2D, D2H), created on first use
+    cudaStream_t hs_down = nullptr;
 
     ~Plan();
     const KernelDesc &kernel() const { return *cands[chosen]; }

@@ -53,6 +53,8 @@ void check_cuda(cudaError_t e, const char *what) {
 Plan::~Plan() {
     for (void *b : ws)
         if (b) cudaFree(b);
+    if (hs_up) cudaStreamDestroy(hs_up);
+    if (hs_down) cudaStreamDestroy(hs_down);
 }
 
 // Algorithmic HBM bytes per written point (reading R10):
@@ -404,11 +406,26 @@ void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int
     }
 }
 
+// End-to-end apply with host buffers, pipelined over z-chunks of the output
+// (concurrent streaming, applied to the PCIe link): chunk c's input
+// planes [z0-R, z1+R) go up on one copy stream, its sweep runs on `stream`,
+// and its output planes come down on a second copy stream, so the H2D of
+// chunk c+1, the sweep of chunk c and the D2H of chunk c-1 overlap (PCIe is
+// full duplex).  Only planes not yet resident are copied, so every input byte
+// crosses the link once.  Outputs come back as the interior box only, so the
+// host ring is untouched.  Synchronous: returns after the last D2H.
 void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int n1, const double *s, int ns,
                 cudaStream_t stream, int64_t *h2d, int64_t *d2h) {
-    const int64_t elems = p->dims[0] * p->dims[1] * p->dims[2];
+    const int64_t nz = p->dims[0], ny = p->dims[1], nx = p->dims[2];
+    const int64_t elems = nz * ny * nx, plane = ny * nx;
     if (n3 != p->n3() || n1 != p->n1() || ns != p->ns()) throw Error(SDAG_ERR_INVALID_ARG, "argument counts");
+    if (n3 > 0 && !h3) throw Error(SDAG_ERR_INVALID_ARG, "null host arrays");
+    for (int f = 0; f < n3; f++)
+        if (!h3[f]) throw Error(SDAG_ERR_INVALID_ARG, "null host array #" + std::to_string(f));
+    for (int f = 0; f < n1; f++)
+        if (!h1 || !h1[f]) throw Error(SDAG_ERR_INVALID_ARG, "null host 1D array #" + std::to_string(f));
     DeviceGuard g(p);
+    std::lock_guard<std::mutex> hl(p->host_mu);
     {
         std::lock_guard<std::mutex> lk(p->mu);
         if (p->ws.empty()) {
@@ -422,43 +439,95 @@ void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int
                 p->ws_bytes[n3 + f] = size_t(p->dims[p->st.formal(ArgKind::Array1D, f).axis]) * 8;
                 check_cuda(cudaMalloc(&p->ws[n3 + f], p->ws_bytes[n3 + f]), "cudaMalloc(workspace)");
             }
+            check_cuda(cudaStreamCreateWithFlags(&p->hs_up, cudaStreamNonBlocking), "cudaStreamCreate");
+            check_cuda(cudaStreamCreateWithFlags(&p->hs_down, cudaStreamNonBlocking), "cudaStreamCreate");
         }
     }
-    int64_t up = 0, down = 0;
+    const int64_t R = p->an.radius[0];
+    const int64_t zlo = p->lo[0], zhi = p->hi[0];
+    // chunks of >= 8 planes (and >= 2R_z so the halo share stays small), at most 16
+    const int64_t nzi = std::max<int64_t>(0, zhi - zlo);
+    const int64_t nch = std::max<int64_t>(1, std::min<int64_t>(16, nzi / std::max<int64_t>(8, 2 * R)));
+    const int64_t zc = nzi > 0 ? (nzi + nch - 1) / nch : 0;
+
     std::vector<double *> d3(n3);
     std::vector<const double *> d1(n1);
-    for (int f = 0; f < n3; f++) {
-        d3[f] = static_cast<double *>(p->ws[f]);
-        const Role r = p->st.formal(ArgKind::Array3D, f).role;
-        if (r == Role::In || r == Role::InOut) {
-            check_cuda(cudaMemcpyAsync(d3[f], h3[f], p->ws_bytes[f], cudaMemcpyHostToDevice, stream), "H2D");
-            up += int64_t(p->ws_bytes[f]);
+    for (int f = 0; f < n3; f++) d3[f] = static_cast<double *>(p->ws[f]);
+    for (int f = 0; f < n1; f++) d1[f] = static_cast<const double *>(p->ws[n3 + f]);
+    const KernelDesc &k = pick_kernel(p, d3.data(), nx);
+
+    std::vector<cudaEvent_t> evs;
+    auto event = [&]() {
+        cudaEvent_t e;
+        check_cuda(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "cudaEventCreate");
+        evs.push_back(e);
+        return e;
+    };
+    struct Cleanup {
+        std::vector<cudaEvent_t> &e;
+        ~Cleanup() {
+            for (cudaEvent_t x : e) cudaEventDestroy(x);
         }
-    }
+    } cleanup{evs};
+
+    int64_t up = 0, down = 0;
+    cudaEvent_t e0 = event();
+    check_cuda(cudaEventRecord(e0, stream), "cudaEventRecord");  // respect the caller's stream order
+    check_cuda(cudaStreamWaitEvent(p->hs_up, e0, 0), "cudaStreamWaitEvent");
+    check_cuda(cudaStreamWaitEvent(p->hs_down, e0, 0), "cudaStreamWaitEvent");
     for (int f = 0; f < n1; f++) {
-        d1[f] = static_cast<const double *>(p->ws[n3 + f]);
-        check_cuda(cudaMemcpyAsync(p->ws[n3 + f], h1[f], p->ws_bytes[n3 + f], cudaMemcpyHostToDevice, stream), "H2D");
+        check_cuda(cudaMemcpyAsync(p->ws[n3 + f], h1[f], p->ws_bytes[n3 + f], cudaMemcpyHostToDevice, p->hs_up), "H2D");
         up += int64_t(p->ws_bytes[n3 + f]);
     }
-    apply(p, d3.data(), n3, d1.data(), n1, s, ns, 1, stream);
-    // copy back the written interior box only, so the host ring stays untouched
-    for (int f = 0; f < n3; f++) {
-        const Role r = p->st.formal(ArgKind::Array3D, f).role;
-        if (r != Role::Out && r != Role::InOut) continue;
-        cudaMemcpy3DParms c;
-        std::memset(&c, 0, sizeof c);
-        const size_t nx = size_t(p->dims[2]), ny = size_t(p->dims[1]), nz = size_t(p->dims[0]);
-        c.srcPtr = make_cudaPitchedPtr(d3[f], nx * 8, nx, ny);
-        c.dstPtr = make_cudaPitchedPtr(h3[f], nx * 8, nx, ny);
-        c.srcPos = make_cudaPos(size_t(p->lo[2]) * 8, size_t(p->lo[1]), size_t(p->lo[0]));
-        c.dstPos = c.srcPos;
-        c.extent = make_cudaExtent(size_t(p->hi[2] - p->lo[2]) * 8, size_t(p->hi[1] - p->lo[1]),
-                                   size_t(p->hi[0] - p->lo[0]));
-        c.kind = cudaMemcpyDeviceToHost;
-        (void)nz;
-        check_cuda(cudaMemcpy3DAsync(&c, stream), "D2H");
-        down += int64_t(c.extent.width) * int64_t(c.extent.height) * int64_t(c.extent.depth);
+    auto upload = [&](int64_t z0, int64_t z1) {  // planes [z0, z1) of every input / inout
+        if (z1 <= z0) return;
+        for (int f = 0; f < n3; f++) {
+            const Role r = p->st.formal(ArgKind::Array3D, f).role;
+            if (r != Role::In && r != Role::InOut) continue;
+            const size_t off = size_t(z0 * plane), cnt = size_t((z1 - z0) * plane);
+            check_cuda(cudaMemcpyAsync(d3[f] + off, h3[f] + off, cnt * 8, cudaMemcpyHostToDevice, p->hs_up), "H2D");
+            up += int64_t(cnt * 8);
+        }
+    };
+    auto download = [&](int64_t z0, int64_t z1) {  // interior box of output planes [z0, z1)
+        for (int f = 0; f < n3; f++) {
+            const Role r = p->st.formal(ArgKind::Array3D, f).role;
+            if (r != Role::Out && r != Role::InOut) continue;
+            cudaMemcpy3DParms c;
+            std::memset(&c, 0, sizeof c);
+            c.srcPtr = make_cudaPitchedPtr(d3[f], size_t(nx) * 8, size_t(nx), size_t(ny));
+            c.dstPtr = make_cudaPitchedPtr(h3[f], size_t(nx) * 8, size_t(nx), size_t(ny));
+            c.srcPos = make_cudaPos(size_t(p->lo[2]) * 8, size_t(p->lo[1]), size_t(z0));
+            c.dstPos = c.srcPos;
+            c.extent = make_cudaExtent(size_t(p->hi[2] - p->lo[2]) * 8, size_t(p->hi[1] - p->lo[1]), size_t(z1 - z0));
+            c.kind = cudaMemcpyDeviceToHost;
+            check_cuda(cudaMemcpy3DAsync(&c, p->hs_down), "D2H");
+            down += int64_t(c.extent.width) * int64_t(c.extent.height) * int64_t(c.extent.depth);
+        }
+    };
+    int64_t resident = 0;  // input planes [0, resident) are on the device
+    for (int64_t c = 0; c < nch && zc > 0; c++) {
+        const int64_t z0 = zlo + c * zc, z1 = std::min(zhi, z0 + zc);
+        if (z0 >= z1) break;
+        const int64_t need = (c == nch - 1) ? nz : std::min(nz, z1 + R);
+        upload(resident, need);
+        resident = std::max(resident, need);
+        cudaEvent_t ein = event();
+        check_cuda(cudaEventRecord(ein, p->hs_up), "cudaEventRecord");
+        check_cuda(cudaStreamWaitEvent(stream, ein, 0), "cudaStreamWaitEvent");
+        plan_launch(p, k, d3.data(), d1.data(), s, 1, z0, z1, stream);
+        cudaEvent_t ec = event();
+        check_cuda(cudaEventRecord(ec, stream), "cudaEventRecord");
+        check_cuda(cudaStreamWaitEvent(p->hs_down, ec, 0), "cudaStreamWaitEvent");
+        download(z0, z1);
     }
+    if (zc == 0) upload(0, nz);  // degenerate grid: nothing to compute, nothing written
+    cudaEvent_t eend = event();
+    check_cuda(cudaEventRecord(eend, p->hs_down), "cudaEventRecord");
+    check_cuda(cudaStreamWaitEvent(stream, eend, 0), "cudaStreamWaitEvent");
+    cudaEvent_t eup = event();
+    check_cuda(cudaEventRecord(eup, p->hs_up), "cudaEventRecord");
+    check_cuda(cudaStreamWaitEvent(stream, eup, 0), "cudaStreamWaitEvent");
     check_cuda(cudaStreamSynchronize(stream), "cudaStreamSynchronize");
     if (h2d) *h2d = up;
     if (d2h) *d2h = down;
