@@ -140,8 +140,8 @@ static int occupancy_of(const Plan *p, const KernelDesc &k) {
     return std::min(bySmem, byThreads);
 }
 
-// z-chunking (concurrent streaming): pick the number of chunks that
-// minimises waves x (chunk + per-unit overhead) for this grid.
+// z-chunking (concurrent streaming): pick the number of z-chunks
+// per xy tile that minimises the modelled time of the grid.
 static void geometry(const Plan *p, const KernelDesc &k, int batch, int64_t klo, int64_t khi, const int64_t *lo,
                      const int64_t *hi, Launch &L) {
     const int64_t nzi = khi - klo;
@@ -150,21 +150,31 @@ static void geometry(const Plan *p, const KernelDesc &k, int batch, int64_t klo,
     const int64_t tiles = int64_t(L.tiles_x) * L.tiles_y * batch;
     const int occ = occupancy_of(p, k);
     const int64_t slots = int64_t(p->sm_count) * occ;
-    // per-unit overhead in plane times: the re-streamed z-halo (2 R_z planes,
-    // mostly L2 hits) plus the ring fill.  With >= 3 resident CTAs per SM a
-    // CTA's ring fill overlaps its neighbours' steady state, and small units
-    // balance the tail better (measured with tools/chunk_sweep.py on B200:
-    // batched 64^3 Jacobi 0.117 -> 0.109 ms, 512^3 27-point 0.360 -> 0.351 ms;
-    // the 1-2 CTA/SM kernels (lap25, hypterm, rhs4) keep the full refill term)
-    const double ovh = occ >= 3 ? double(k.rzr) : double(2 * k.rzr + 2);
+    // Cost model (measured with tools/chunk_sweep.py on B200):
+    //  * one resident CTA per SM: equal units run in lock-step waves, so the
+    //    cost is waves x (chunk + z-halo 2H + ring refill 2) -- hypterm prefers 3
+    //    chunks (3.95 waves) to 4 (5.3 waves) by 10 %;
+    //  * >= 2 resident CTAs: slots backfill as units finish, so the cost is the
+    //    fluid work units x (chunk + 2H) / slots plus one unit of tail --
+    //    small units trim the tail (batched 64^3 Jacobi 0.117 -> 0.109 ms,
+    //    512^3 27-point 0.361 -> 0.341 ms) while the z-halo re-streamed per
+    //    unit keeps radius-4 stencils at long chunks (lap25: 8 chunks of 63).
+    // z-halo planes a unit streams beyond its chunk, per side (radius x fused sweeps)
+    const int64_t halo = int64_t(std::max(k.rz, k.rzr)) * std::max(1, k.tsteps);
     double best = 1e300;
     int bestn = 1;
     const int maxn = int(std::min<int64_t>(nzi, std::max<int64_t>(1, 65535 / std::max(batch, 1))));
     for (int n = 1; n <= std::min(maxn, 512); n++) {
         const int64_t zc = (nzi + n - 1) / n;
         const int64_t units = tiles * ((nzi + zc - 1) / zc);
-        const double waves = double((units + slots - 1) / slots);
-        const double cost = waves * (double(zc) + ovh);
+        double cost;
+        if (occ <= 1) {
+            const double waves = double((units + slots - 1) / slots);
+            cost = waves * double(zc + 2 * halo + 2);
+        } else {
+            const double tu = double(zc + 2 * halo);
+            cost = double(units) * tu / double(slots) + tu;
+        }
         if (cost < best - 1e-9) {
             best = cost;
             bestn = n;
