@@ -68,6 +68,7 @@ typedef enum sdag_status {
 } sdag_status;
 
 typedef struct sdag_plan_s *sdag_plan;
+typedef struct sdag_program_s *sdag_program;
 typedef struct sdag_dist_s *sdag_dist;
 typedef struct CUstream_st *sdag_stream; /* == cudaStream_t; NULL = legacy default stream */
 
@@ -148,6 +149,36 @@ sdag_status sdag_apply(sdag_plan plan, double *const *arrays3d, int32_t n3d, con
 sdag_status sdag_apply_batched(sdag_plan plan, int32_t batch, double *const *arrays3d, int32_t n3d,
                                const double *const *arrays1d, int32_t n1d, const double *scalars,
                                int32_t nscalars, sdag_stream stream);
+
+/*
+ * Multi-stencil programs (Fig 3c): a spec
+ * with several `stencil` definitions and calls in sequence.  Each call is one
+ * stage, planned like sdag_plan_create (registered kernel or NVRTC-generated
+ * one); sdag_program_apply enqueues the stages in call order on `stream`, each
+ * a full sweep over its own interior that sees the arrays as the earlier
+ * stages left them (a later stage may read an earlier stage's output at any
+ * offset).  sdag_plan_create rejects such specs with SDAG_ERR_UNSUPPORTED.
+ *
+ * Arguments are the program's DECLARED arrays and scalars that some call
+ * binds, in declaration order (the generated host function's parameters,
+ * P:439-441) -- not a stencil's formal order.  Roles (sdag_program_arg, 3D):
+ * 0 in (read before any stage writes it), 1 out (first touched by a write;
+ * intermediates read by later stages are out and caller-owned), 2 inout
+ * (read, then written by a later stage).  Strings live as long as the program.
+ * sdag_program_stage returns a BORROWED plan handle for stage s (info,
+ * describe, variants, args); never pass it to sdag_plan_destroy.
+ * sdag_program_apply validates every stage (counts, nulls, output aliasing
+ * within a stage) before enqueuing anything; errors as sdag_apply.
+ */
+sdag_status sdag_program_create(const char *spec, const int64_t dims[3], const sdag_plan_opts *opts,
+                                sdag_program *out);
+sdag_status sdag_program_info(sdag_program prog, int32_t *n_stages, int32_t *n3d, int32_t *n1d, int32_t *nscalars);
+sdag_status sdag_program_arg(sdag_program prog, int32_t kind, int32_t idx, const char **name, int32_t *role);
+sdag_status sdag_program_stage(sdag_program prog, int32_t s, sdag_plan *out);
+sdag_status sdag_program_apply(sdag_program prog, int32_t batch, double *const *arrays3d, int32_t n3d,
+                               const double *const *arrays1d, int32_t n1d, const double *scalars, int32_t nscalars,
+                               sdag_stream stream);
+void sdag_program_destroy(sdag_program prog);
 
 /*
  * a6: T sweeps ping-pong (Fig 1a; time loop P:380-381) of a plan

@@ -393,3 +393,77 @@ def roles(text):
             continue
         out[f] = ("inout" if f in read_before else "out") if f in written else "in"
     return out
+
+
+# ---------------------------------------------------------------------------
+# Multi-stencil programs (Fig 3c): several stencil
+# definitions and calls in sequence.  The plain definition: the calls run in
+# program order, each one a complete evaluation of its stencil (above) on the
+# arrays as the previous calls left them; a call's written grids replace the
+# bound arrays' interiors.  Programs take declared names (not formals).
+# ---------------------------------------------------------------------------
+
+def _split_program(text):
+    """-> (prelude text, {stencil name: definition text}, [(name, call text)])"""
+    t = _strip(text)
+    defs, calls, prelude = {}, [], []
+    i = 0
+    stmt_start = 0
+    while i < len(t):
+        m = re.match(r"\s*stencil\s+([A-Za-z_]\w*)", t[i:])
+        if m and (i == 0 or not (t[i - 1].isalnum() or t[i - 1] == "_")) and t[i:i + m.end()].strip().startswith("stencil"):
+            j = t.index("{", i)
+            depth, k = 0, j
+            while True:
+                depth += (t[k] == "{") - (t[k] == "}")
+                k += 1
+                if depth == 0:
+                    break
+            defs[m.group(1)] = t[i:k]
+            i = k
+            stmt_start = i
+            continue
+        if t[i] == ";":
+            stmt = t[stmt_start:i + 1]
+            cm = re.match(r"\s*([A-Za-z_]\w*)\s*\(", stmt)
+            if cm and cm.group(1) in defs:
+                calls.append((cm.group(1), stmt))
+            else:
+                prelude.append(stmt)
+            stmt_start = i + 1
+        i += 1
+    return "\n".join(prelude), defs, calls
+
+
+def program_stages(text):
+    """[(single-stencil spec text, {formal: declared name})] in call order."""
+    prelude, defs, calls = _split_program(text)
+    if not calls:
+        if len(defs) != 1:
+            raise ValueError("several stencils but no call")
+        (name, d), = defs.items()
+        one = prelude + "\n" + d
+        return [(one, {f: f for f in Spec(one).formals})]
+    out = []
+    for name, c in calls:
+        one = prelude + "\n" + defs[name] + "\n" + c
+        sp = Spec(one)
+        out.append((one, _bind(sp)))
+    return out
+
+
+def evaluate_program(text, dims, arrays, scalars, absmode=False):
+    """Evaluate a program; arrays / scalars keyed by DECLARED names.  Returns a
+    dict declared name -> grid for every array some stage wrote.  With
+    absmode=True every stage runs in abs mode on the abs-mode results of the
+    earlier stages (the error-gate bound of the composition, reading R13)."""
+    state = {k: np.array(v, dtype=np.float64, copy=True) for k, v in arrays.items()}
+    written = set()
+    for one, bind in program_stages(text):
+        fa = {f: state[a] for f, a in bind.items() if a in state}
+        fs = {f: scalars[a] for f, a in bind.items() if a in scalars}
+        res = evaluate(one, dims, fa, fs, absmode=absmode)
+        for f, g in res.items():
+            state[bind[f]] = g
+            written.add(bind[f])
+    return {k: state[k] for k in written}

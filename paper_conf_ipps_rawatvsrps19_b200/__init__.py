@@ -21,7 +21,7 @@ import os
 from . import _capi
 from ._capi import PlanInfo, PlanOpts, SDAG_DEVICE_CURRENT, SDAG_DEVICE_NONE
 
-__all__ = ["Plan", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "slab_partition2", "slab_halo2", "nccl_unique_id",
+__all__ = ["Plan", "Program", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "slab_partition2", "slab_halo2", "nccl_unique_id",
            "nccl_comm_create", "nccl_comm_destroy", "launch_count", "fp64_peak", "version", "SPEC_DIR"]
 
 SPEC_DIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "specs")
@@ -213,6 +213,72 @@ class Plan:
         _check(self._L.sdag_apply_host(self._h, _arr(p3), len(p3), _arr(p1), len(p1), s, ns, _stream_handle(stream),
                                        ctypes.byref(up), ctypes.byref(down)))
         return up.value, down.value
+
+
+class Program:
+    """A multi-stencil program (several stencils and calls, Fig 3c): one planned
+    stage per call, applied in call order.  Arguments are the declared arrays
+    and scalars in declaration order (sdag_program_*)."""
+
+    def __init__(self, spec: str, dims, order=-1, device=None, tune=False, batch=1, variant=None):
+        self._L = _capi.lib()
+        self._h = ctypes.c_void_p()
+        d = (ctypes.c_int64 * 3)(*[int(x) for x in dims])
+        o = _opts(order, device, tune, batch, variant, True)
+        _check(self._L.sdag_program_create(spec.encode(), d, ctypes.byref(o), ctypes.byref(self._h)))
+
+    def close(self):
+        if self._h:
+            self._L.sdag_program_destroy(self._h)
+        self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    @property
+    def counts(self) -> dict:
+        n, a3, a1, sc = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+        _check(self._L.sdag_program_info(self._h, ctypes.byref(n), ctypes.byref(a3), ctypes.byref(a1),
+                                         ctypes.byref(sc)))
+        return {"n_stages": n.value, "n_arrays3d": a3.value, "n_arrays1d": a1.value, "n_scalars": sc.value}
+
+    def args(self):
+        """[(kind, index, name, role_or_axis)] in declaration order per kind."""
+        c = self.counts
+        out = []
+        for kind, n in ((0, c["n_arrays3d"]), (1, c["n_arrays1d"]), (2, c["n_scalars"])):
+            for q in range(n):
+                nm, r = ctypes.c_char_p(), ctypes.c_int32()
+                _check(self._L.sdag_program_arg(self._h, kind, q, ctypes.byref(nm), ctypes.byref(r)))
+                out.append((kind, q, nm.value.decode(), r.value))
+        return out
+
+    def arg_names(self, kind: int):
+        return [a[2] for a in self.args() if a[0] == kind]
+
+    def stage(self, s: int) -> Plan:
+        """Borrowed plan of stage s (introspection only; owned by the program)."""
+        h = ctypes.c_void_p()
+        _check(self._L.sdag_program_stage(self._h, int(s), ctypes.byref(h)))
+        p = Plan._borrow(h.value)
+        p._program = self  # keep the owner alive
+        return p
+
+    def apply(self, arrays3d, arrays1d=(), scalars=(), stream=None, batch=1):
+        p3 = [_ptr(t, "grid array") for t in arrays3d]
+        p1 = [_ptr(t, "1D array") for t in arrays1d]
+        s, ns = _scal(scalars)
+        _check(self._L.sdag_program_apply(self._h, int(batch), _arr(p3), len(p3), _arr(p1), len(p1), s, ns,
+                                          _stream_handle(stream)))
 
 
 def fusion_schedule(f, T: int):

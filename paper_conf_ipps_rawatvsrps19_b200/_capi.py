@@ -62,6 +62,14 @@ def lib():
             "sdag_apply_iterated": (S, [P, c_void_p, c_void_p, c_i32, c_dblp, c_i32, P]),
             "sdag_apply_host": (S, [P, ctypes.POINTER(c_void_p), c_i32, ctypes.POINTER(c_void_p), c_i32, c_dblp,
                                     c_i32, P, c_i64p, c_i64p]),
+            "sdag_program_create": (S, [c_char_p, c_i64p, ctypes.POINTER(PlanOpts), ctypes.POINTER(P)]),
+            "sdag_program_info": (S, [P, ctypes.POINTER(c_i32), ctypes.POINTER(c_i32), ctypes.POINTER(c_i32),
+                                      ctypes.POINTER(c_i32)]),
+            "sdag_program_arg": (S, [P, c_i32, c_i32, ctypes.POINTER(c_char_p), ctypes.POINTER(c_i32)]),
+            "sdag_program_stage": (S, [P, c_i32, ctypes.POINTER(P)]),
+            "sdag_program_apply": (S, [P, c_i32, ctypes.POINTER(c_void_p), c_i32, ctypes.POINTER(c_void_p), c_i32,
+                                       c_dblp, c_i32, P]),
+            "sdag_program_destroy": (None, [P]),
             "sdag_fusion_schedule": (S, [c_dblp, c_i32, c_i32, ctypes.POINTER(c_i32), c_i32,
                                          ctypes.POINTER(c_i32), c_dblp]),
             "sdag_slab_partition": (S, [c_i64, c_i32, c_i32, c_i32, c_i64p]),
@@ -100,6 +108,8 @@ def lib():
 EXPORTED = [
     "sdag_plan_opts_init", "sdag_plan_create", "sdag_plan_info_get", "sdag_plan_arg", "sdag_plan_variant_name",
     "sdag_plan_describe", "sdag_plan_destroy", "sdag_apply", "sdag_apply_batched", "sdag_apply_iterated",
+    "sdag_program_create", "sdag_program_info", "sdag_program_arg", "sdag_program_stage", "sdag_program_apply",
+    "sdag_program_destroy",
     "sdag_apply_host", "sdag_fusion_schedule", "sdag_slab_partition", "sdag_slab_halo",
     "sdag_slab_partition2", "sdag_slab_halo2", "sdag_nccl_get_unique_id", "sdag_nccl_comm_create",
     "sdag_nccl_comm_destroy", "sdag_dist_create", "sdag_dist_layout", "sdag_dist_local_plan", "sdag_dist_apply",

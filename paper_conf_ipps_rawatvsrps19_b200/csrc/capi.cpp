@@ -102,6 +102,70 @@ void sdag_plan_destroy(sdag_plan plan) {
     delete plan;
 }
 
+// ---- multi-stencil programs (Fig 3c) ----
+
+static sdag::Program *G(sdag_program g) {
+    if (!g || !g->g) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null program");
+    return g->g;
+}
+
+sdag_status sdag_program_create(const char *spec, const int64_t dims[3], const sdag_plan_opts *opts,
+                                sdag_program *out) {
+    return guard([&] {
+        if (!spec || !dims || !out) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null argument");
+        *out = nullptr;
+        sdag_plan_opts o;
+        sdag_plan_opts_init(&o);
+        if (opts) o = *opts;
+        sdag::Program *g = sdag::program_create(spec, dims, o);
+        *out = new sdag_program_s{g};
+    });
+}
+
+sdag_status sdag_program_info(sdag_program prog, int32_t *n_stages, int32_t *n3d, int32_t *n1d, int32_t *nscalars) {
+    return guard([&] {
+        sdag::Program *g = G(prog);
+        if (n_stages) *n_stages = int32_t(g->stages.size());
+        if (n3d) *n3d = g->n_of(sdag::ArgKind::Array3D);
+        if (n1d) *n1d = g->n_of(sdag::ArgKind::Array1D);
+        if (nscalars) *nscalars = g->n_of(sdag::ArgKind::Scalar);
+    });
+}
+
+sdag_status sdag_program_arg(sdag_program prog, int32_t kind, int32_t idx, const char **name, int32_t *role) {
+    return guard([&] {
+        sdag::Program *g = G(prog);
+        if (kind < 0 || kind > 2) throw sdag::Error(SDAG_ERR_INVALID_ARG, "kind must be 0, 1 or 2");
+        const auto k = static_cast<sdag::ArgKind>(kind);
+        if (idx < 0 || idx >= g->n_of(k)) throw sdag::Error(SDAG_ERR_INVALID_ARG, "index out of range");
+        const sdag::ProgramArg &a = g->arg(k, idx);
+        if (name) *name = a.name.c_str();
+        if (role) *role = (k == sdag::ArgKind::Array3D) ? int32_t(a.role) : (k == sdag::ArgKind::Array1D ? a.axis : -1);
+    });
+}
+
+sdag_status sdag_program_stage(sdag_program prog, int32_t s, sdag_plan *out) {
+    return guard([&] {
+        sdag::Program *g = G(prog);
+        if (!out) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null out");
+        if (s < 0 || s >= int32_t(g->stages.size())) throw sdag::Error(SDAG_ERR_INVALID_ARG, "stage out of range");
+        *out = g->handles[s];
+    });
+}
+
+sdag_status sdag_program_apply(sdag_program prog, int32_t batch, double *const *a3, int32_t n3,
+                               const double *const *a1, int32_t n1, const double *s, int32_t ns, sdag_stream stream) {
+    return guard([&] {
+        sdag::program_apply(G(prog), a3, n3, a1, n1, s, ns, batch, reinterpret_cast<cudaStream_t>(stream));
+    });
+}
+
+void sdag_program_destroy(sdag_program prog) {
+    if (!prog) return;
+    delete prog->g;
+    delete prog;
+}
+
 sdag_status sdag_apply(sdag_plan plan, double *const *a3, int32_t n3, const double *const *a1, int32_t n1,
                        const double *s, int32_t ns, sdag_stream stream) {
     return guard([&] { sdag::apply(P(plan), a3, n3, a1, n1, s, ns, 1, reinterpret_cast<cudaStream_t>(stream)); });

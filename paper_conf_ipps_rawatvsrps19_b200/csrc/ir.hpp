@@ -102,8 +102,26 @@ struct Error : std::runtime_error {
     Error(int st, const std::string &m) : std::runtime_error(m), status(st) {}
 };
 
-// a1: parse the DSL text into a resolved Stencil (throws Error).
+// a1: parse the DSL text into a resolved Stencil (throws Error).  Specs with
+// several stencil definitions or calls are programs: UNSUPPORTED here.
 Stencil parse_spec(const std::string &text);
+
+// A multi-stencil program (Fig 3c): one resolved Stencil per
+// call, in call order; every stage is a full sweep over its own interior and
+// sees the arrays as the previous stages left them.
+struct ProgramArg {
+    std::string name;  // declared name
+    ArgKind kind = ArgKind::Scalar;
+    int kind_index = -1;  // position among program arguments of the same kind (declaration order)
+    int axis = -1;        // 1D arrays
+    Role role = Role::Unused;  // program-level (filled by the planner)
+};
+struct ProgramIR {
+    std::vector<Stencil> stages;
+    std::vector<ProgramArg> args;        // declared names bound by some stage, declaration order
+    std::vector<std::vector<int>> map;   // map[s][formal position] = index into args
+};
+ProgramIR parse_program(const std::string &text);
 // a2: analyse (throws Error for UNSUPPORTED / SEMANTIC findings).
 Analysis analyse(const Stencil &st);
 // canonical, name-free serialisation used to match registered DAGs

@@ -69,6 +69,26 @@ struct Plan {
 
 // planner (runtime.cu)
 Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_plan_opts &o);
+Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &o);
+
+// A multi-stencil program (Fig 3c): one plan per call, run in call order on
+// one stream (program.cpp).  Arguments are the program's declared arrays and
+// scalars in declaration order; stage s's formal q is program argument map[s][q].
+struct Program {
+    ProgramIR ir;
+    std::vector<std::unique_ptr<Plan>> stages;
+    std::vector<sdag_plan_s *> handles;  // borrowed per-stage handles (sdag_program_stage)
+    int n_of(ArgKind k) const {
+        int n = 0;
+        for (auto &a : ir.args) n += (a.kind == k);
+        return n;
+    }
+    const ProgramArg &arg(ArgKind k, int idx) const;
+    ~Program();
+};
+Program *program_create(const std::string &spec, const int64_t dims[3], const sdag_plan_opts &o);
+void program_apply(Program *g, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns,
+                   int batch, cudaStream_t stream);
 void plan_fill_info(Plan *p, sdag_plan_info *info);
 
 // sweep launch over output planes [klo, khi) of each problem (clipped to the
@@ -78,6 +98,9 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *arrays3d, const do
                  const int64_t *dims_override = nullptr, const int64_t *zr = nullptr);
 void apply(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns, int batch,
            cudaStream_t stream);
+// the argument checks of apply (counts, nulls, output aliasing), nothing enqueued
+void plan_validate(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns,
+                   int batch);
 std::vector<int> fusion_schedule(const double *f, int maxdeg, int T);
 void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int ns, cudaStream_t stream);
 void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int n1, const double *s, int ns,
@@ -96,7 +119,10 @@ double measure_fp64_peak(cudaStream_t stream);
 
 }  // namespace sdag
 
-// the opaque C handle (include/sdag.h) wraps a Plan
+// the opaque C handles (include/sdag.h) wrap a Plan / a Program
 struct sdag_plan_s {
     sdag::Plan *p;
+};
+struct sdag_program_s {
+    sdag::Program *g;
 };

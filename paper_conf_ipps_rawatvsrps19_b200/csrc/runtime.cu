@@ -336,6 +336,13 @@ struct DeviceGuard {
     }
 };
 
+void plan_validate(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns,
+                   int batch) {
+    if (batch < 1) throw Error(SDAG_ERR_INVALID_ARG, "batch must be >= 1");
+    validate_arrays(p, a3, n3, a1, n1, ns, p->dims[0] * p->dims[1] * p->dims[2] * batch);
+    if (ns > 0 && !s) throw Error(SDAG_ERR_INVALID_ARG, "null scalars");
+}
+
 void apply(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns, int batch,
            cudaStream_t stream) {
     if (batch < 1) throw Error(SDAG_ERR_INVALID_ARG, "batch must be >= 1");
@@ -550,8 +557,12 @@ void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int
 static void time_candidates(Plan *p);
 
 Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_plan_opts &o) {
+    return plan_create_from(parse_spec(spec), dims, o);  // a1
+}
+
+Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &o) {
     std::unique_ptr<Plan> p(new Plan());
-    p->st = parse_spec(spec);                 // a1
+    p->st = std::move(st);
     p->an = analyse(p->st);                   // a2
     const int nit = int(p->st.iterators.size());
     for (int a = 0; a < 3; a++) {

@@ -10,6 +10,9 @@
 //           | '#pragma' ... EOL
 //           | 'stencil' ID '(' ids ')' '{' { stmt } '}'
 //           | ID '(' ids ')' ';'              call, positional binding
+// A spec with one stencil and at most one call is a plan (parse_spec); several
+// stencil definitions and calls in sequence are a program (Fig 3c, P:1349-1368;
+// parse_program), each call one stage.
 //   stmt   := '#assign' ... EOL
 //           | ['double'] lhs ('='|'+='|'-='|'*='|'/=') expr ';'
 //   expr   := C precedence over + - * / unary-, parentheses, literals,
@@ -166,16 +169,29 @@ struct Parser {
     std::map<std::string, Decl> decls;
     std::vector<std::string> decl_order;
 
-    bool have_stencil = false;
-    std::string sname;
-    std::vector<std::string> formals;
-    std::vector<RawStmt> body;
-    Pragma pragma, pending_pragma;
+    struct Def {  // one `stencil` definition
+        std::string name;
+        std::vector<std::string> formals;
+        std::vector<RawStmt> body;
+        Pragma pragma;
+        Assign assign;
+        int line = 0, col = 0;
+    };
+    struct Call {  // one call, actuals bound positionally
+        std::string name;
+        std::vector<std::string> actuals;
+        int line = 0, col = 0;
+    };
+    std::vector<Def> defs;
+    std::vector<Call> calls;
+    Pragma pending_pragma;
     bool have_pending_pragma = false;
-    Assign assign;
-    int n_stencils = 0, n_calls = 0;
-    std::vector<std::string> actuals;
-    int call_line = 0, call_col = 0;
+
+    const Def *def_of(const std::string &n) const {
+        for (auto &d : defs)
+            if (d.name == n) return &d;
+        return nullptr;
+    }
 
     const Tok &cur() const { return tk[p]; }
     bool is(const char *s) const { return (cur().k == Tok::Punct || cur().k == Tok::Id) && cur().s == s; }
@@ -266,23 +282,23 @@ struct Parser {
             expect(";");
         } else if (t.s == "stencil") {
             p++;
-            n_stencils++;
-            if (n_stencils > 1)
-                fail(SDAG_ERR_UNSUPPORTED, t.line, t.col,
-                     "multi-stencil programs (Fig 3c) are not on the hot path yet");
-            have_stencil = true;
-            sname = ident();
+            Def d;
+            d.line = cur().line;
+            d.col = cur().col;
+            d.name = ident();
+            if (def_of(d.name)) fail(SDAG_ERR_SEMANTIC, d.line, d.col, "stencil '" + d.name + "' defined twice");
             if (have_pending_pragma) {
-                pragma = pending_pragma;
+                d.pragma = pending_pragma;
                 have_pending_pragma = false;
             }
             expect("(");
             if (!is(")")) {
-                do formals.push_back(ident());
+                do d.formals.push_back(ident());
                 while (is(",") && (p++, true));
             }
             expect(")");
             expect("{");
+            defs.push_back(std::move(d));
             while (!is("}")) {
                 if (cur().k == Tok::End) err("unterminated stencil body");
                 stmt();
@@ -290,21 +306,21 @@ struct Parser {
             expect("}");
         } else {
             // call: name(actuals);
-            int l = t.line, c = t.col;
-            std::string n = ident();
-            if (!is("(")) fail(SDAG_ERR_PARSE, l, c, "unknown statement '" + n + "'");
+            Call cl;
+            cl.line = t.line;
+            cl.col = t.col;
+            cl.name = ident();
+            if (!is("(")) fail(SDAG_ERR_PARSE, cl.line, cl.col, "unknown statement '" + cl.name + "'");
             p++;
-            n_calls++;
-            if (n_calls > 1) fail(SDAG_ERR_UNSUPPORTED, l, c, "more than one stencil call");
-            if (!have_stencil || n != sname) fail(SDAG_ERR_SEMANTIC, l, c, "call of undefined stencil '" + n + "'");
-            call_line = l;
-            call_col = c;
+            if (!def_of(cl.name))
+                fail(SDAG_ERR_SEMANTIC, cl.line, cl.col, "call of undefined stencil '" + cl.name + "'");
             if (!is(")")) {
-                do actuals.push_back(ident());
+                do cl.actuals.push_back(ident());
                 while (is(",") && (p++, true));
             }
             expect(")");
             expect(";");
+            calls.push_back(std::move(cl));
         }
     }
 
@@ -362,7 +378,7 @@ struct Parser {
             if (sub[q].s != "(") fail(SDAG_ERR_PARSE, t.line, t.col, "#assign: expected (");
             q++;
             while (sub[q].k == Tok::Id) {
-                (kind == "shmem" ? assign.shmem : assign.gmem).push_back(sub[q++].s);
+                (kind == "shmem" ? defs.back().assign.shmem : defs.back().assign.gmem).push_back(sub[q++].s);
                 if (sub[q].s == ",") q++;
             }
             if (sub[q].s != ")") fail(SDAG_ERR_PARSE, t.line, t.col, "#assign: expected )");
@@ -426,7 +442,7 @@ struct Parser {
         if (s.declares && s.op != "=") err("declaration needs '='");
         s.rhs = expr();
         expect(";");
-        body.push_back(std::move(s));
+        defs.back().body.push_back(std::move(s));
     }
 
     std::unique_ptr<Raw> expr() {
@@ -505,13 +521,15 @@ struct Parser {
 
 struct Resolver {
     const Parser &P;
+    const Parser::Def &D;
+    const Parser::Call *C;  // null: the definition evaluated on its own formals
     Stencil &S;
     std::map<std::string, int> formal_of;  // formal name -> index in S.formals
     std::map<std::string, int> temp_of;
     std::set<std::string> temp_assigned;
     int n_iter = 0;
 
-    Resolver(const Parser &p, Stencil &s) : P(p), S(s) {}
+    Resolver(const Parser &p, const Parser::Def &d, const Parser::Call *c, Stencil &s) : P(p), D(d), C(c), S(s) {}
 
     int iter_pos(const std::string &it) const {
         for (int q = 0; q < n_iter; q++)
@@ -615,27 +633,27 @@ struct Resolver {
     void run() {
         n_iter = (int)P.iters.size();
         if (n_iter == 0) fail(SDAG_ERR_SEMANTIC, 1, 1, "no 'iterator' declaration");
-        if (!P.have_stencil) fail(SDAG_ERR_SEMANTIC, 1, 1, "no 'stencil' function");
-        S.name = P.sname;
+        S.name = D.name;
         S.iterators = P.iters;
         S.parameters = P.params;
-        S.pragma = P.pragma;
-        S.assign = P.assign;
-        S.has_call = P.n_calls == 1;
-        if (S.has_call && P.actuals.size() != P.formals.size())
-            fail(SDAG_ERR_SEMANTIC, P.call_line, P.call_col,
-                 "call passes " + std::to_string(P.actuals.size()) + " arguments, stencil takes " +
-                     std::to_string(P.formals.size()));
+        S.pragma = D.pragma;
+        S.assign = D.assign;
+        S.has_call = C != nullptr;
+        if (C && C->actuals.size() != D.formals.size())
+            fail(SDAG_ERR_SEMANTIC, C->line, C->col,
+                 "call passes " + std::to_string(C->actuals.size()) + " arguments, stencil takes " +
+                     std::to_string(D.formals.size()));
         int cnt[3] = {0, 0, 0};
         std::set<std::string> seen;
-        for (size_t q = 0; q < P.formals.size(); q++) {
+        for (size_t q = 0; q < D.formals.size(); q++) {
             Formal f;
-            f.name = P.formals[q];
-            if (!seen.insert(f.name).second) fail(SDAG_ERR_SEMANTIC, 1, 1, "duplicate formal '" + f.name + "'");
-            f.actual = S.has_call ? P.actuals[q] : f.name;
+            f.name = D.formals[q];
+            if (!seen.insert(f.name).second)
+                fail(SDAG_ERR_SEMANTIC, D.line, D.col, "duplicate formal '" + f.name + "'");
+            f.actual = C ? C->actuals[q] : f.name;
             auto d = P.decls.find(f.actual);
             if (d == P.decls.end())
-                fail(SDAG_ERR_SEMANTIC, S.has_call ? P.call_line : 1, S.has_call ? P.call_col : 1,
+                fail(SDAG_ERR_SEMANTIC, C ? C->line : D.line, C ? C->col : D.col,
                      "argument '" + f.actual + "' is not declared");
             size_t nd = d->second.dims.size();
             if (nd == 0) f.kind = ArgKind::Scalar;
@@ -649,7 +667,7 @@ struct Resolver {
             formal_of[f.name] = (int)S.formals.size();
             S.formals.push_back(f);
         }
-        for (auto &rs : P.body) {
+        for (auto &rs : D.body) {
             Statement st;
             st.line = rs.line;
             st.declares = rs.declares;
@@ -704,7 +722,7 @@ struct Resolver {
             }
             S.stmts.push_back(st);
         }
-        if (S.stmts.empty()) fail(SDAG_ERR_SEMANTIC, 1, 1, "empty stencil body");
+        if (S.stmts.empty()) fail(SDAG_ERR_SEMANTIC, D.line, D.col, "empty stencil body");
         for (auto &f : S.formals)
             if (f.kind == ArgKind::Array1D && f.axis < 0) f.axis = 2;  // unused 1D array
     }
@@ -716,10 +734,64 @@ Stencil parse_spec(const std::string &text) {
     Parser P;
     P.tk = lex(text);
     P.parse();
+    if (P.defs.empty()) fail(SDAG_ERR_SEMANTIC, 1, 1, "no 'stencil' function");
+    if (P.defs.size() > 1 || P.calls.size() > 1) {
+        const int l = P.defs.size() > 1 ? P.defs[1].line : P.calls[1].line;
+        const int c = P.defs.size() > 1 ? P.defs[1].col : P.calls[1].col;
+        fail(SDAG_ERR_UNSUPPORTED, l, c,
+             "multi-stencil program (Fig 3c): plan it with sdag_program_create, one stage per call");
+    }
     Stencil S;
-    Resolver R(P, S);
+    Resolver R(P, P.defs[0], P.calls.empty() ? nullptr : &P.calls[0], S);
     R.run();
     return S;
+}
+
+ProgramIR parse_program(const std::string &text) {
+    Parser P;
+    P.tk = lex(text);
+    P.parse();
+    if (P.defs.empty()) fail(SDAG_ERR_SEMANTIC, 1, 1, "no 'stencil' function");
+    ProgramIR G;
+    if (P.calls.empty()) {
+        if (P.defs.size() > 1)
+            fail(SDAG_ERR_SEMANTIC, P.defs[1].line, P.defs[1].col, "several stencils but no call to order them");
+        G.stages.emplace_back();
+        Resolver R(P, P.defs[0], nullptr, G.stages.back());
+        R.run();
+    } else {
+        for (const auto &cl : P.calls) {
+            G.stages.emplace_back();
+            Resolver R(P, *P.def_of(cl.name), &cl, G.stages.back());
+            R.run();
+        }
+    }
+    // program arguments: the declared names some stage binds, in declaration order
+    std::set<std::string> used;
+    for (const auto &st : G.stages)
+        for (const auto &f : st.formals) used.insert(f.actual);
+    int cnt[3] = {0, 0, 0};
+    for (const auto &n : P.decl_order) {
+        if (!used.count(n)) continue;
+        ProgramArg a;
+        a.name = n;
+        for (const auto &st : G.stages)
+            for (const auto &f : st.formals)
+                if (f.actual == n) {
+                    a.kind = f.kind;
+                    if (f.kind == ArgKind::Array1D) a.axis = f.axis;
+                }
+        a.kind_index = cnt[int(a.kind)]++;
+        G.args.push_back(a);
+    }
+    for (const auto &st : G.stages) {
+        std::vector<int> m;
+        for (const auto &f : st.formals)
+            for (size_t q = 0; q < G.args.size(); q++)
+                if (G.args[q].name == f.actual) m.push_back(int(q));
+        G.map.push_back(m);
+    }
+    return G;
 }
 
 }  // namespace sdag
