@@ -22,15 +22,23 @@
 namespace sdag {
 namespace dev {
 
-template <int GX, int GY, int UY, int PF, int UX = 2>
+// ODD = false: the box starts 2 columns left of the region (ML = 2), a patch
+//   starts at an even smem column and its 3-point row window [c-1, c+UX] is read
+//   as UX/2 + 2 aligned pairs, two of them half used;
+// ODD = true: the box starts 3 columns left (ML = 3, tile origin even, box
+//   origin still 16-B aligned), a patch starts at an odd smem column, and its
+//   window [c-1, c+UX] is exactly UX/2 + 1 aligned pairs -- a third fewer
+//   shared-memory reads per fold for UX = 2 (the fused kernel is bound by them).
+template <int GX, int GY, int UY, int PF, int UX = 2, bool ODD = false>
 struct Fuse2Geo {
-    static constexpr int ML = 2;                 // box x margin (region - 2): 16-B alignment
+    static constexpr int ML = ODD ? 3 : 2;       // box x margin (region - ML): 16-B alignment of the box origin
     static constexpr int NTX = GX / UX, NTY = GY / UY, THREADS = NTX * NTY, NWARPS = (THREADS + 31) / 32;
-    static constexpr int PX = GX + 4, PY = GY + 2, PLANE = PX * PY;  // input box / S1 plane layout
+    static constexpr int PX = GX + (ODD ? 6 : 4), PY = GY + 2, PLANE = PX * PY;  // input box / S1 plane layout
     static constexpr int PLANE_AL = ((PLANE * 8 + 127) / 128) * 128 / 8;
     static constexpr int NS = 1 + PF;
     static constexpr int SMEM = (NS + 2) * PLANE_AL * 8 + 2 * NS * 8;
-    static constexpr int NW = UX + 4;            // row window [cx, cx+UX+4) in smem columns (16-B aligned)
+    static constexpr int NW = ODD ? UX + 2 : UX + 4;  // row window in smem columns (16-B aligned start)
+    static constexpr int W0 = ODD ? ML - 1 : 0;       // window start relative to the patch's smem column - ML
     static_assert((UX == 2 || UX == 4) && GX % UX == 0 && GY % UY == 0, "region");
     static_assert(PX <= 256 && PY <= 256, "TMA box");
 };
@@ -38,11 +46,11 @@ struct Fuse2Geo {
 // UX = 2 or 4 output columns per thread: the row window of a UX-wide patch is
 // UX+4 doubles read with (UX+4)/2 128-bit loads, so UX = 4 cuts the fold's
 // shared-memory reads per point from 1.5 to 1 LDS.128 per row.
-template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2>
-__global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX>::THREADS, MINB)
+template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2, bool ODD = false>
+__global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MINB)
     sdag_box27x2(const __grid_constant__ SweepArgs a) {
-    using G = Fuse2Geo<GX, GY, UY, PF, UX>;
-    constexpr int PX = G::PX, NS = G::NS, PAL = G::PLANE_AL, ML = G::ML, NW = G::NW;
+    using G = Fuse2Geo<GX, GY, UY, PF, UX, ODD>;
+    constexpr int PX = G::PX, NS = G::NS, PAL = G::PLANE_AL, ML = G::ML, NW = G::NW, W0 = G::W0;
     constexpr int TX = GX - 2, TY = GY - 2;  // output tile
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -118,7 +126,7 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX>::THREADS, MINB)
         double w[UY + 2][NW];
 #pragma unroll
         for (int r = 0; r < UY + 2; r++) {
-            const double *rp = pl + (cy + r) * PX + cx;
+            const double *rp = pl + (cy + r) * PX + cx + W0;
 #pragma unroll
             for (int c = 0; c < NW / 2; c++) {
                 const double2 v = *reinterpret_cast<const double2 *>(rp + 2 * c);
@@ -130,7 +138,7 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX>::THREADS, MINB)
         for (int py = 0; py < UY; py++)
 #pragma unroll
             for (int px = 0; px < UX; px++) {
-                const int c = ML + px;
+                const int c = ML - W0 + px;  // the patch point's column in the window
                 const double s0 = w[py + 1][c];
                 const double s1 = (w[py + 1][c - 1] + w[py + 1][c + 1]) + (w[py][c] + w[py + 2][c]);
                 const double s2 = (w[py][c - 1] + w[py][c + 1]) + (w[py + 2][c - 1] + w[py + 2][c + 1]);
@@ -165,8 +173,15 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX>::THREADS, MINB)
                 A1[py][px] = s0[py][px];
             }
 #pragma unroll
-            for (int px = 0; px < UX; px += 2)
-                *reinterpret_cast<double2 *>(s1 + (cy + py + 1) * PX + cx + ML + px) = make_double2(v[px], v[px + 1]);
+            for (int px = 0; px < UX; px += 2) {
+                double *q = s1 + (cy + py + 1) * PX + cx + ML + px;
+                if constexpr (ODD) {
+                    q[0] = v[px];
+                    q[1] = v[px + 1];
+                } else {
+                    *reinterpret_cast<double2 *>(q) = make_double2(v[px], v[px + 1]);
+                }
+            }
         }
         __syncthreads();  // sweep-1 plane j is complete in shared memory
         if (j < kb - 1) continue;  // sweep-2 state starts at sweep-1 plane kb-1

@@ -236,18 +236,19 @@ KernelDesc make_star2_desc(const char *dag, int prio) {
     v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, QM, 1>(DAG, PRIO))
 
 // two fused sweeps of the 27-point smoother (fuse2.cuh), TMA only
-template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2>
+template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2, bool ODD = false>
 KernelDesc make_fuse2_desc(const char *dag, int prio) {
-    using G = dev::Fuse2Geo<GX, GY, UY, PF, UX>;
+    using G = dev::Fuse2Geo<GX, GY, UY, PF, UX, ODD>;
     KernelDesc d;
     d.dag = dag;
     char buf[96];
+    const char *tag = ODD ? "fuse2o" : "fuse2";
     if (MINB > 1)
-        std::snprintf(buf, sizeof buf, "fuse2_tma_%dx%d_u%dx%d_pf%d_mb%d", GX - 2, GY - 2, UX, UY, PF, MINB);
+        std::snprintf(buf, sizeof buf, "%s_tma_%dx%d_u%dx%d_pf%d_mb%d", tag, GX - 2, GY - 2, UX, UY, PF, MINB);
     else
-        std::snprintf(buf, sizeof buf, "fuse2_tma_%dx%d_u%dx%d_pf%d", GX - 2, GY - 2, UX, UY, PF);
+        std::snprintf(buf, sizeof buf, "%s_tma_%dx%d_u%dx%d_pf%d", tag, GX - 2, GY - 2, UX, UY, PF);
     d.variant = buf;
-    d.fn = reinterpret_cast<const void *>(&dev::sdag_box27x2<GX, GY, UY, PF, MINB, UX>);
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_box27x2<GX, GY, UY, PF, MINB, UX, ODD>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = GX - 2;
@@ -260,7 +261,7 @@ KernelDesc make_fuse2_desc(const char *dag, int prio) {
     d.nout = 1;
     d.rz = 1;
     d.ry = 2;  // TMA box (GY+2) = ty + 2*ry
-    d.rx = 3;  // TMA box (GX+4) = tx + 2*rx, origin tile-3 (even)
+    d.rx = ODD ? 4 : 3;  // TMA box PX = tx + 2*rx, origin tile - rx (even)
     d.rzr = 2;
     d.prio = prio;
     d.tsteps = 2;

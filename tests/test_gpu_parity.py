@@ -384,7 +384,9 @@ def test_full_size_smooth27_iterated_sampled():
 
 
 FUSED = ["fuse2_tma_62x14_u2x2_pf2_mb2", "fuse2_tma_30x14_u2x2_pf2_mb3", "fuse2_tma_126x14_u2x4_pf2", "fuse2_tma_62x30_u2x2_pf2",
-         "fuse2_tma_126x14_u2x2_pf2", "fuse2_tma_62x14_u4x2_pf2"]
+         "fuse2_tma_126x14_u2x2_pf2", "fuse2_tma_62x14_u4x2_pf2",
+         "fuse2o_tma_62x14_u2x2_pf2_mb2", "fuse2o_tma_30x14_u2x2_pf2_mb3", "fuse2o_tma_126x14_u2x4_pf2",
+         "fuse2o_tma_62x14_u4x2_pf2_mb2"]
 
 
 @pytest.mark.parametrize("variant", FUSED)

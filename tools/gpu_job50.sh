@@ -1,0 +1,4 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -m gpu --timeout 600 -k "fusion or loopback or smooth27" > gpurun_out/pt_fuse.log 2>&1; echo "exit $?" >> gpurun_out/pt_fuse.log
+timeout 600 python bench.py --config smooth27 > gpurun_out/bench_s27.json 2> gpurun_out/bench_s27.err
