@@ -1,4 +1,5 @@
-// fuse2.cuh -- temporal fusion of two sweeps of the 27-point smoother
+// fuse2.cuh -- temporal fusion of two sweeps of the 27-point smoother (and of
+// Listing 1's 7-point Jacobi, FORM 1)
 // (NEXT-1: the paper's fusion for arbitrary time iterations, with
 // overlapped tiling, Fig 1b).
 //
@@ -46,7 +47,11 @@ struct Fuse2Geo {
 // UX = 2 or 4 output columns per thread: the row window of a UX-wide patch is
 // UX+4 doubles read with (UX+4)/2 128-bit loads, so UX = 4 cuts the fold's
 // shared-memory reads per point from 1.5 to 1 LDS.128 per row.
-template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2, bool ODD = false>
+// FORM 0: the 27-point smoother (scalars w0..w3, nu);
+// FORM 1: Listing 1's 7-point Jacobi (scalars h2inv, a, b), the paper's
+//   7pt-smoother of Table I / Table II, in box27's retimed FORM 1:
+//   T_k = s1_k - 6 s0_k + s0_{k-1}, B[k] = a A[k] - (b h2inv)(T_k + s0_{k+1}).
+template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2, bool ODD = false, int FORM = 0>
 __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MINB)
     sdag_box27x2(const __grid_constant__ SweepArgs a) {
     using G = Fuse2Geo<GX, GY, UY, PF, UX, ODD>;
@@ -96,6 +101,7 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
         if (p <= plast) issue(p);
 
     const double w0 = a.s[0], w1 = a.s[1], w2 = a.s[2], w3 = a.s[3], nu = a.s[4];
+    const double ja = a.s[1], jc = a.s[2] * a.s[0];  // FORM 1: a, c = b*h2inv
 
     // region point (cy+py, cx+px) -> global (ry0+cy+py, rx0+cx+px); x/y ring flags
     bool ringxy[UY][UX];
@@ -141,9 +147,14 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
                 const int c = ML - W0 + px;  // the patch point's column in the window
                 const double s0 = w[py + 1][c];
                 const double s1 = (w[py + 1][c - 1] + w[py + 1][c + 1]) + (w[py][c] + w[py + 2][c]);
-                const double s2 = (w[py][c - 1] + w[py][c + 1]) + (w[py + 2][c - 1] + w[py + 2][c + 1]);
-                cc[py][px] = fma(w2, s2, fma(w1, s1, w0 * s0));
-                uu[py][px] = fma(w3, s2, fma(w2, s1, w1 * s0));
+                if constexpr (FORM == 0) {
+                    const double s2 = (w[py][c - 1] + w[py][c + 1]) + (w[py + 2][c - 1] + w[py + 2][c + 1]);
+                    cc[py][px] = fma(w2, s2, fma(w1, s1, w0 * s0));
+                    uu[py][px] = fma(w3, s2, fma(w2, s1, w1 * s0));
+                } else {
+                    cc[py][px] = s1;  // in-plane face sum
+                    uu[py][px] = 0.0;
+                }
                 s0v[py][px] = s0;
             }
     };
@@ -166,10 +177,15 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
             double v[UX];
 #pragma unroll
             for (int px = 0; px < UX; px++) {
-                v[px] = fma(nu, T1[py][px] + uu[py][px], A1[py][px]);
+                if constexpr (FORM == 0) {
+                    v[px] = fma(nu, T1[py][px] + uu[py][px], A1[py][px]);
+                    T1[py][px] = U1[py][px] + cc[py][px];
+                    U1[py][px] = uu[py][px];
+                } else {
+                    v[px] = ja * A1[py][px] - jc * (T1[py][px] + s0[py][px]);
+                    T1[py][px] = fma(-6.0, s0[py][px], cc[py][px] + A1[py][px]);
+                }
                 if (zring || ringxy[py][px]) v[px] = A1[py][px];  // ring: not updated by sweep 1
-                T1[py][px] = U1[py][px] + cc[py][px];
-                U1[py][px] = uu[py][px];
                 A1[py][px] = s0[py][px];
             }
 #pragma unroll
@@ -194,9 +210,14 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
             double res[UX];
 #pragma unroll
             for (int px = 0; px < UX; px++) {
-                res[px] = fma(nu, T2[py][px] + uu[py][px], A2[py][px]);
-                T2[py][px] = U2[py][px] + cc[py][px];
-                U2[py][px] = uu[py][px];
+                if constexpr (FORM == 0) {
+                    res[px] = fma(nu, T2[py][px] + uu[py][px], A2[py][px]);
+                    T2[py][px] = U2[py][px] + cc[py][px];
+                    U2[py][px] = uu[py][px];
+                } else {
+                    res[px] = ja * A2[py][px] - jc * (T2[py][px] + s0[py][px]);
+                    T2[py][px] = fma(-6.0, s0[py][px], cc[py][px] + A2[py][px]);
+                }
                 A2[py][px] = s0[py][px];
             }
             const int ry = cy + py, gj = ry0 + ry;

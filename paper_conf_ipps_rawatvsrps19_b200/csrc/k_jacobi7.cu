@@ -11,5 +11,14 @@ void add_kernels_jacobi7(std::vector<KernelDesc> &v) {
     SDAG_CROSS_PAIR(v, "jacobi7", 64, 64, 8, 3, 5);
     SDAG_STAR_PAIR(v, Jacobi7Star, "jacobi7", 64, 16, 2, 6, 6);
     SDAG_PAIR(v, Jacobi7, "jacobi7", 64, 16, 1, 4, 2, 10);
+    // temporal fusion for apply_iterated (NEXT-1; the paper's 7pt-smoother,
+    // Table II): two sweeps per launch, overlapped tiles.  The cross stencil's
+    // y-neighbour rows need only the patch's own (aligned) pair, so the
+    // even-aligned layout wins here (tools/table2_sweep.py, 1024^3 T=12:
+    // 2.03 ms/sweep vs 2.19 odd-aligned vs 3.04 unfused)
+    v.push_back(make_fuse2_desc<64, 16, 2, 2, 2, 2, false, 1>("jacobi7", 20));
+    v.push_back(make_fuse2_desc<64, 16, 2, 2, 2, 2, true, 1>("jacobi7", 21));
+    v.push_back(make_fuse2_desc<32, 16, 2, 2, 3, 2, true, 1>("jacobi7", 22));
+    v.push_back(make_fuse2_desc<128, 16, 4, 2, 1, 2, true, 1>("jacobi7", 23));
 }
 }  // namespace sdag

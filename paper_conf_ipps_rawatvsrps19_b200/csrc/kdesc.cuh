@@ -236,7 +236,7 @@ KernelDesc make_star2_desc(const char *dag, int prio) {
     v.push_back(make_star_desc<dev::BODY, TX, TY, UY, PF, true, QM, 1>(DAG, PRIO))
 
 // two fused sweeps of the 27-point smoother (fuse2.cuh), TMA only
-template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2, bool ODD = false>
+template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2, bool ODD = false, int FORM = 0>
 KernelDesc make_fuse2_desc(const char *dag, int prio) {
     using G = dev::Fuse2Geo<GX, GY, UY, PF, UX, ODD>;
     KernelDesc d;
@@ -248,7 +248,7 @@ KernelDesc make_fuse2_desc(const char *dag, int prio) {
     else
         std::snprintf(buf, sizeof buf, "%s_tma_%dx%d_u%dx%d_pf%d", tag, GX - 2, GY - 2, UX, UY, PF);
     d.variant = buf;
-    d.fn = reinterpret_cast<const void *>(&dev::sdag_box27x2<GX, GY, UY, PF, MINB, UX, ODD>);
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_box27x2<GX, GY, UY, PF, MINB, UX, ODD, FORM>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = GX - 2;

@@ -420,6 +420,42 @@ def test_temporal_fusion_matches_oracle_and_unfused(variant, dims):
         assert np.array_equal(gf[ring_mask(dims, 1)], A[ring_mask(dims, 1)])
 
 
+FUSED_J7 = ["fuse2o_tma_62x14_u2x2_pf2_mb2", "fuse2o_tma_30x14_u2x2_pf2_mb3", "fuse2o_tma_126x14_u2x4_pf2",
+            "fuse2_tma_62x14_u2x2_pf2_mb2"]
+
+
+def _jacobi7_iter(A, a, b, h2inv, T, absmode=False):
+    """T oracle sweeps, ping-pong with a fixed ring (Fig 1a semantics, reading R1)."""
+    cur = np.array(A, copy=True)
+    for _ in range(T):
+        cur = oracle.jacobi7(cur, a, b, h2inv, absmode=absmode, out=cur.copy())
+    return cur
+
+
+@pytest.mark.parametrize("variant", FUSED_J7)
+@pytest.mark.parametrize("dims", [(26, 30, 40), (9, 70, 260)], ids=lambda d: "x".join(map(str, d)))
+def test_temporal_fusion_jacobi7(variant, dims):
+    """NEXT-1 on Listing 1's 7-point Jacobi (the paper's 7pt-smoother, Table II):
+    two sweeps per launch vs T oracle sweeps, odd and even T, ring untouched."""
+    ins, sc = synth.jacobi7_inputs(dims, cfg="fuse")
+    A = ins["A"]
+    s = [sc["h2inv"], sc["a"], sc["b"]]
+    fused = sdag.Plan(sdag.spec_text("jacobi7"), dims, variant=variant)
+    for T in (1, 2, 5, 6):
+        b0 = torch.from_numpy(A).cuda()
+        b1 = b0.clone()
+        n0 = sdag.launch_count()
+        fused.apply_iterated(b0, b1, T, scalars=s)
+        torch.cuda.synchronize()
+        g = (b0 if T % 2 == 0 else b1).cpu().numpy()
+        # launches flip the ping-pong pair once each, so #launches == T (mod 2)
+        assert sdag.launch_count() - n0 == {1: 1, 2: 2, 5: 3, 6: 4}[T]
+        O = _jacobi7_iter(A, sc["a"], sc["b"], sc["h2inv"], T)
+        Aabs = _jacobi7_iter(np.abs(A), sc["a"], sc["b"], sc["h2inv"], T, absmode=True)
+        assert scaled_err(g, O, Aabs) <= T * TOL
+        assert np.array_equal(g[ring_mask(dims, 1)], A[ring_mask(dims, 1)])
+
+
 def test_temporal_fusion_exact_closed_form():
     """V8 through the fused kernels: integer weights, quadratic input, bit-exact."""
     dims, T = (16, 18, 20), 4
