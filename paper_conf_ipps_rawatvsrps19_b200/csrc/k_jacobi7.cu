@@ -17,8 +17,17 @@ void add_kernels_jacobi7(std::vector<KernelDesc> &v) {
     // even-aligned layout wins here (tools/table2_sweep.py, 1024^3 T=12:
     // 2.03 ms/sweep vs 2.19 odd-aligned vs 3.04 unfused)
     v.push_back(make_fuse2_desc<64, 16, 2, 2, 2, 2, false, 1>("jacobi7", 20));
+    v.back().fhint = 1.29;  // f(2) measured at 1024^3 (tools/table2_sweep.py --all)
     v.push_back(make_fuse2_desc<64, 16, 2, 2, 2, 2, true, 1>("jacobi7", 21));
     v.push_back(make_fuse2_desc<32, 16, 2, 2, 3, 2, true, 1>("jacobi7", 22));
     v.push_back(make_fuse2_desc<128, 16, 4, 2, 1, 2, true, 1>("jacobi7", 23));
+    // fusion degrees 3 and 4 (fuseN.cuh): the paper's Table II / Fig 4 sweep
+    v.push_back(make_fuseN_desc<3, 64, 32, 2, 2, 1, 2, false, 1>("jacobi7", 40));
+    v.back().fhint = 1.96;  // f(3): 0.65 per sweep, the cusp (f(2)/2 = 0.64)
+    v.push_back(make_fuseN_desc<3, 64, 32, 2, 2, 1, 2, true, 1>("jacobi7", 41));
+    v.push_back(make_fuseN_desc<3, 128, 16, 2, 2, 1, 2, false, 1>("jacobi7", 42));
+    v.push_back(make_fuseN_desc<4, 64, 32, 2, 2, 1, 2, false, 1>("jacobi7", 43));
+    v.back().fhint = 3.17;  // f(4): 0.79 per sweep
+    v.push_back(make_fuseN_desc<4, 64, 16, 2, 2, 2, 2, false, 1>("jacobi7", 44));
 }
 }  // namespace sdag

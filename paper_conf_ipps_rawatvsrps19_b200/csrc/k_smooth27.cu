@@ -14,6 +14,7 @@ void add_kernels_smooth27(std::vector<KernelDesc> &v) {
     // tools/fusion_sweep.py at 1024^3, T=12: odd-aligned 62x14 2.27 ms/sweep,
     // even-aligned 62x14 2.51, unfused 2.77
     v.push_back(make_fuse2_desc<64, 16, 2, 2, 2, 2, true>("smooth27", 20));  // mb2: 2 CTAs/SM need <= 128 registers
+    v.back().fhint = 1.69;  // f(2) measured at 1024^3 (tools/table2_sweep.py --all)
     v.push_back(make_fuse2_desc<32, 16, 2, 2, 3, 2, true>("smooth27", 21));
     v.push_back(make_fuse2_desc<64, 16, 2, 2, 2>("smooth27", 22));
     v.push_back(make_fuse2_desc<32, 16, 2, 2, 3>("smooth27", 23));
@@ -23,5 +24,13 @@ void add_kernels_smooth27(std::vector<KernelDesc> &v) {
     v.push_back(make_fuse2_desc<128, 16, 2, 2>("smooth27", 27));
     v.push_back(make_fuse2_desc<64, 16, 2, 2, 2, 4, true>("smooth27", 28));
     v.push_back(make_fuse2_desc<64, 16, 2, 2, 1, 4>("smooth27", 29));  // 4-wide patch: bank-conflicted, kept for comparison
+    // fusion degrees 3 and 4 (fuseN.cuh): the paper's Table II / Fig 4 sweep
+    v.push_back(make_fuseN_desc<3, 64, 32, 2, 2, 1, 2, false, 0>("smooth27", 40));
+    v.back().fhint = 3.12;  // f(3): 1.04 per sweep -- past the cusp (shared-memory bound folds)
+    v.push_back(make_fuseN_desc<3, 64, 32, 2, 2, 1, 2, true, 0>("smooth27", 41));
+    v.push_back(make_fuseN_desc<3, 128, 16, 2, 2, 1, 2, false, 0>("smooth27", 42));
+    v.push_back(make_fuseN_desc<4, 64, 32, 2, 2, 1, 2, false, 0>("smooth27", 43));
+    v.back().fhint = 4.96;  // f(4): 1.24 per sweep
+    v.push_back(make_fuseN_desc<4, 64, 16, 2, 2, 2, 2, false, 0>("smooth27", 44));
 }
 }  // namespace sdag

@@ -8,6 +8,7 @@
 #include "kernels.hpp"
 #include "box27.cuh"
 #include "fuse2.cuh"
+#include "fuseN.cuh"
 #include "hyp.cuh"
 #include "rhs4.cuh"
 #include "star.cuh"
@@ -265,6 +266,37 @@ KernelDesc make_fuse2_desc(const char *dag, int prio) {
     d.rzr = 2;
     d.prio = prio;
     d.tsteps = 2;
+    return d;
+}
+
+// NT >= 2 fused sweeps (fuseN.cuh), TMA only
+template <int NT, int GX, int GY, int UY, int PF, int MINB, int UX, bool ODD, int FORM>
+KernelDesc make_fuseN_desc(const char *dag, int prio) {
+    using G = dev::FuseNGeo<NT, GX, GY, UY, PF, UX, ODD>;
+    constexpr int H = NT - 1;
+    KernelDesc d;
+    d.dag = dag;
+    char buf[96];
+    std::snprintf(buf, sizeof buf, "fuse%d%s_tma_%dx%d_u%dx%d_pf%d_mb%d", NT, ODD ? "o" : "", GX - 2 * H, GY - 2 * H,
+                  UX, UY, PF, MINB);
+    d.variant = buf;
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_boxfuse<NT, GX, GY, UY, PF, MINB, UX, ODD, FORM>);
+    d.threads = G::THREADS;
+    d.smem = G::SMEM;
+    d.tx = GX - 2 * H;
+    d.ty = GY - 2 * H;
+    d.ux = UX;
+    d.uy = UY;
+    d.pf = PF;
+    d.tma = true;
+    d.nin = 1;
+    d.nout = 1;
+    d.rz = 1;
+    d.ry = NT;          // TMA box (GY + 2) = ty + 2 * ry
+    d.rx = H + G::ML;   // TMA box PX = tx + 2 * rx, origin tile - rx (even)
+    d.rzr = 1;
+    d.prio = prio;
+    d.tsteps = NT;
     return d;
 }
 

@@ -19,6 +19,7 @@ struct KernelDesc {
     int rz = 0, ry = 0, rx = 0, rzr = 0;  // body radius and shared-memory ring z-window
     int prio = 0;                         // heuristic preference (lower first)
     int tsteps = 1;                       // sweeps fused per launch (temporal fusion, NEXT-1)
+    double fhint = 0.0;                   // measured f(x): launch cost / one sweep (0 = generic estimate)
     void *cufn = nullptr;                 // CUfunction of an NVRTC-compiled kernel (jit.cu); fn is then null
 };
 

@@ -160,7 +160,7 @@ static void geometry(const Plan *p, const KernelDesc &k, int batch, int64_t klo,
     //    512^3 27-point 0.361 -> 0.341 ms) while the z-halo re-streamed per
     //    unit keeps radius-4 stencils at long chunks (lap25: 8 chunks of 63).
     // z-halo planes a unit streams beyond its chunk, per side (radius x fused sweeps)
-    const int64_t halo = int64_t(std::max(k.rz, k.rzr)) * std::max(1, k.tsteps);
+    const int64_t halo = k.tsteps > 1 ? int64_t(k.rz) * k.tsteps : int64_t(std::max(k.rz, k.rzr));
     double best = 1e300;
     int bestn = 1;
     const int maxn = int(std::min<int64_t>(nzi, std::max<int64_t>(1, 65535 / std::max(batch, 1))));
@@ -673,7 +673,8 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
     // bandwidth-bound stencil -- an x-sweep launch moves the data of one sweep
     // plus overlapped-tiling overhead; replaced by measured times when tune=1
     p->fcost[1] = 1.0;
-    for (const KernelDesc *f : p->fused) p->fcost[f->tsteps] = 1.0 + 0.15 * (f->tsteps - 1);
+    for (const KernelDesc *f : p->fused)  // first (preferred) kernel of each degree
+        if (p->fcost[f->tsteps] == 0.0) p->fcost[f->tsteps] = f->fhint > 0.0 ? f->fhint : 1.0 + 0.15 * (f->tsteps - 1);
     std::stable_sort(p->cands.begin(), p->cands.end(),
                      [](const KernelDesc *a, const KernelDesc *b) { return a->prio < b->prio; });
     if (p->cands.empty()) throw Error(SDAG_ERR_UNSUPPORTED, "no kernel variant fits this plan");

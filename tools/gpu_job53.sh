@@ -1,0 +1,5 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -m gpu --timeout 600 -k "fusion or loopback" > gpurun_out/pt_fN.log 2>&1; echo "exit $?" >> gpurun_out/pt_fN.log
+timeout 900 python tools/table2_sweep.py --n 1024 --reps 2 > gpurun_out/table2_def1024.jsonl 2>&1
+timeout 600 python bench.py --config smooth27 > gpurun_out/bench_s27.json 2> gpurun_out/bench_s27.err

@@ -45,11 +45,21 @@ def main():
     ap.add_argument("--n", type=int, default=512)
     ap.add_argument("--T", type=int, default=12)
     ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--all", action="store_true", help="also time every fused kernel forced")
     a = ap.parse_args()
     dims = (a.n, a.n, a.n)
     for name in ("jacobi7", "smooth27"):
-        for kw in ({"fusion": False}, {}, {"tune": True}):
-            print(json.dumps(run(name, dims, a.T, a.reps, **kw)), flush=True)
+        cfgs = [{"fusion": False}, {}, {"tune": True}]
+        if a.all:
+            base = sdag.Plan(sdag.spec_text(name), dims)
+            for ln in base.describe().splitlines():
+                if "temporal fusion" in ln:
+                    cfgs += [{"variant": w} for w in ln.split(":", 1)[1].split() if w.startswith("fuse")]
+        for kw in cfgs:
+            rec = run(name, dims, a.T, a.reps, **kw)
+            if "variant" in kw:
+                rec["fused_kernel"] = kw["variant"]
+            print(json.dumps(rec), flush=True)
 
 
 if __name__ == "__main__":
