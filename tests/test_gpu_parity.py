@@ -256,6 +256,44 @@ def test_loopback_slabs_bitwise_equal_single_gpu(name, gdims, T, tt, P):
         assert np.array_equal(got, ref[z0:z0 + n]), f"rank {r} of {P}"
 
 
+@pytest.mark.parametrize("variant,tt", [("fuse3_tma_60x28_u2x2_pf2_mb1", 3), ("fuse4_tma_58x26_u2x2_pf2_mb1", 4)])
+@pytest.mark.parametrize("P", [1, 2, 3])
+def test_loopback_slabs_fusion_degree(variant, tt, P):
+    """NEXT-1 x a7: slabs with ghost depth tt R_z run the forced tt-sweep kernel
+    (one exchange of tt R_z planes per launch) bit-identical to one GPU."""
+    name, gdims, T = "smooth27", (46, 34, 66), 12
+    case = make_case(name, gdims, cfg="slab")
+    A = case["inputs"][0]
+    s = case["s"]
+    spec = sdag.spec_text(name)
+    full = sdag.Plan(spec, gdims, variant=variant)
+    b0 = torch.from_numpy(A).cuda()
+    b1 = b0.clone()
+    full.apply_iterated(b0, b1, T, scalars=s)
+    ref = (b0 if T % 2 == 0 else b1).cpu().numpy()
+    dists = [sdag.Dist(spec, gdims, r, P, time_tile=tt, variant=variant) for r in range(P)]
+    bufs0, bufs1 = [], []
+    for d in dists:
+        (nza, ny, nx), g0 = d.layout()
+        loc = np.zeros((nza, ny, nx))
+        lo, hi = max(g0, 0), min(g0 + nza, gdims[0])
+        loc[lo - g0:hi - g0] = A[lo:hi]
+        bufs0.append(torch.from_numpy(loc).cuda())
+        bufs1.append(torch.from_numpy(loc.copy()).cuda())
+    sdag.Dist.apply_iterated_loopback(dists, bufs0, bufs1, T, scalars=s)
+    torch.cuda.synchronize()
+    res = bufs0 if T % 2 == 0 else bufs1
+    for r, d in enumerate(dists):
+        part = sdag.slab_partition2(gdims[0], RADIUS[name], tt, P, r)
+        (nza, ny, nx), g0 = d.layout()
+        z0, n = part["z0"], part["nz_own"]
+        got = res[r].cpu().numpy()[z0 - g0:z0 - g0 + n]
+        assert np.array_equal(got, ref[z0:z0 + n]), f"rank {r} of {P}"
+    O = oracle.smooth27_iter(A, s[:4], s[4], T)
+    Aabs = oracle.smooth27_iter(np.abs(A), np.abs(s[:4]), s[4], T, absmode=True)
+    assert scaled_err(ref, O, Aabs) <= T * TOL
+
+
 def test_full_size_lap25_sampled():
     """BASELINE config 2 (512^3) in the launch configuration bench.py times,
     checked on sampled points the oracle computes one by one."""
