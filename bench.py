@@ -267,6 +267,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--variant", default=None)
     ap.add_argument("--tune", action="store_true")
+    ap.add_argument("--force-dist", action="store_true",
+                    help="take the z-slab/NCCL path even on one rank (plumbing check of the multi-GPU code)")
     ap.add_argument("--config", default="lap25", choices=list(CONFIGS),
                     help="lap25 = the headline line; the others record the remaining BASELINE stencils (N=1)")
     args = ap.parse_args()
@@ -293,11 +295,12 @@ def main():
     spec = sdag.spec_text(name)
     ldims = CONFIGS[name][1]
     gdims = (ldims[0] * world, ldims[1], ldims[2])
-    ins, sc = synth.lap25_inputs(ldims, cfg="cfg2") if world == 1 else (None, dict(synth.LAP25_COEFS))
+    use_dist = world > 1 or args.force_dist
+    ins, sc = synth.lap25_inputs(ldims, cfg="cfg2") if not use_dist else (None, dict(synth.LAP25_COEFS))
     c = [sc[k] for k in ("c0", "c1", "c2", "c3", "c4")]
     stream = torch.cuda.current_stream()
 
-    if world == 1:
+    if not use_dist:
         plan = sdag.Plan(spec, ldims, tune=args.tune, variant=args.variant)
         A = ins["A"]
         dA = torch.from_numpy(A).cuda()
@@ -310,7 +313,8 @@ def main():
             plan.apply(arrays, scalars=c, stream=stream)
     else:
         uid = [sdag.nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(uid, src=0)
+        if dist:
+            dist.broadcast_object_list(uid, src=0)
         comm = sdag.nccl_comm_create(uid[0], world, rank, local)
         dd = sdag.Dist(spec, gdims, rank, world, comm=comm, tune=args.tune, variant=args.variant)
         (nza, ny, nx), g0 = dd.layout()
@@ -357,8 +361,8 @@ def main():
 
     # dominant kernel: the sweep.  N=1: the step is exactly one launch.  N>1: time the
     # local sweep kernel alone (same stream, same launch configuration).
-    kms = ms / max(1, launches) if world == 1 else None
-    if world > 1:
+    kms = ms / max(1, launches) if not use_dist else None
+    if use_dist:
         ka, kb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         lp = dd.plan
         ka.record(stream)
@@ -370,10 +374,10 @@ def main():
     peak, peak_src = load_peaks()
     bytes_launch = info["bytes_per_point"] * info["points"]
     achieved = bytes_launch / (kms * 1e-3) / 1e9
-    traffic = load_traffic(info["variant"], ldims) if world == 1 else None
+    traffic = load_traffic(info["variant"], ldims) if not use_dist else None
 
     e2e = None
-    if not args.no_e2e and world == 1:
+    if not args.no_e2e and not use_dist:
         hA = torch.from_numpy(A).pin_memory().numpy()
         hB = torch.zeros(ldims, dtype=torch.float64).pin_memory().numpy()
         ee = []
@@ -388,7 +392,7 @@ def main():
                "d2h_bytes_per_step": down, "ms_per_step": t_e2e * 1e3}
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu:
+    if rank == 0 and not use_dist and not args.no_cpu:
         cpu = cpu_baseline_lap25(A, c)
 
     if rank == 0:
@@ -397,7 +401,7 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": CONFIGS[name][2], "stencil": name, "grid_per_gpu": list(ldims),
-                       "global_grid": list(gdims), "decomposition": f"z-slabs x{world}" if world > 1 else "none",
+                       "global_grid": list(gdims), "decomposition": f"z-slabs x{world}" if use_dist else "none",
                        "variant": info["variant"], "flops_per_point": flops_pt,
                        "bytes_per_point": info["bytes_per_point"],
                        "l2": "input 1 GiB/GPU > 126 MB L2 (no flush needed)"},
