@@ -82,7 +82,12 @@ typedef struct sdag_plan_opts {
     int32_t device;            /* CUDA ordinal, SDAG_DEVICE_CURRENT or SDAG_DEVICE_NONE    */
     int32_t tune;              /* 0 = heuristic variant choice; 1 = time the candidates at
                                   plan time on scratch buffers (hierarchical autotuning,
-                                  P:1202-1271) -- synchronises the device                  */
+                                  P:1202-1271) -- synchronises the device.  With the
+                                  environment variable SDAG_TUNE_CACHE naming a file, the
+                                  choice (variant, measured f(x), fused-kernel order) is
+                                  appended there per (version, device, DAG, dims, batch,
+                                  fusion) and later tune=1 plans of that shape restore it
+                                  without timing; an unreadable/unwritable file is ignored */
     int32_t batch;             /* independent problems per apply (sdag_apply_batched); >= 1 */
     const char *force_variant; /* NULL, or a variant name from sdag_plan_variant_name()    */
     int32_t fusion;            /* sdag_apply_iterated: 1 = fuse sweeps where a fused kernel

@@ -36,6 +36,7 @@ struct Plan {
     int sm_count = 148;
     int batch_hint = 1;
     int tune = 0;
+    bool tune_cached = false;  // tune=1 result restored from $SDAG_TUNE_CACHE
     std::string force_variant;
 
     // ABI mapping (per 3D formal kind_index): staged-input slot / output slot / inout slot

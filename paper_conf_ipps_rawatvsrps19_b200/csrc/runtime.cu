@@ -5,6 +5,9 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <fstream>
+#include <functional>
+#include <sstream>
 #include <array>
 #include <atomic>
 #include <cmath>
@@ -555,6 +558,8 @@ void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int
 // ---------------------------------------------------------------------------
 
 static void time_candidates(Plan *p);
+static bool tune_cache_load(Plan *p);
+static void tune_cache_store(const Plan *p);
 
 Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_plan_opts &o) {
     return plan_create_from(parse_spec(spec), dims, o);  // a1
@@ -691,12 +696,19 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
             }
         if (p->chosen < 0) throw Error(SDAG_ERR_INVALID_ARG, "unknown variant '" + p->force_variant + "'");
     } else if (p->tune && !p->host_only) {
-        time_candidates(p.get());
+        if (!tune_cache_load(p.get())) {
+            time_candidates(p.get());
+            tune_cache_store(p.get());
+        } else {
+            p->tune_cached = true;
+        }
     }
 
     const KernelDesc &k = p->kernel();
     d << "\n  variant " << k.variant << " (" << k.threads << " threads, " << k.smem << " B smem, ring "
-      << (2 * k.rzr + 1 + k.pf) << " planes)" << (p->tune ? "  [tuned]" : "  [heuristic]") << "\n  candidates:";
+      << (2 * k.rzr + 1 + k.pf) << " planes)"
+      << (p->tune ? (p->tune_cached ? "  [tuned, from $SDAG_TUNE_CACHE]" : "  [tuned]") : "  [heuristic]")
+      << "\n  candidates:";
     for (auto *c : p->cands) d << " " << c->variant;
     if (!p->fused.empty()) {
         d << "\n  temporal fusion (apply_iterated):";
@@ -709,6 +721,77 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
         d << "\n  jit body (NVRTC, sm_100a, into the sweep.cuh skeleton):\n" << jit_body_source(*p, "JitBody", p->an.radius[0]);
     p->describe_text = d.str();
     return p.release();
+}
+
+// ---------------------------------------------------------------------------
+// Persistent tuning cache (NEXT-3): tune=1 results keyed by (library version,
+// device name, canonical DAG, dims, batch) in the text file named by
+// $SDAG_TUNE_CACHE (off when unset).  One line per plan shape:
+//   key \t chosen variant \t f(1..7) \t fused kernels in measured order
+// A hit restores the choice without timing; a miss tunes and appends.
+// ---------------------------------------------------------------------------
+
+static std::string tune_key(const Plan *p) {
+    cudaDeviceProp prop;
+    std::string dev = "?";
+    if (cudaGetDeviceProperties(&prop, p->device) == cudaSuccess) dev = prop.name;
+    else (void)cudaGetLastError();
+    std::ostringstream k;
+    k << sdag_version() << "|" << dev << "|" << std::hash<std::string>{}(canonical_form(p->st)) << "|"
+      << p->dims[0] << "x" << p->dims[1] << "x" << p->dims[2] << "|b" << p->batch_hint << "|f" << p->fusion;
+    return k.str();
+}
+
+static std::mutex g_tune_file_mu;
+
+static bool tune_cache_load(Plan *p) {
+    const char *path = std::getenv("SDAG_TUNE_CACHE");
+    if (!path || !*path) return false;
+    std::lock_guard<std::mutex> lk(g_tune_file_mu);
+    std::ifstream in(path);
+    if (!in) return false;
+    const std::string key = tune_key(p);
+    std::string line, hit;
+    while (std::getline(in, line))
+        if (line.compare(0, key.size() + 1, key + "\t") == 0) hit = line;  // last entry wins
+    if (hit.empty()) return false;
+    std::vector<std::string> col;
+    std::stringstream ss(hit);
+    for (std::string c; std::getline(ss, c, '\t');) col.push_back(c);
+    if (col.size() < 3) return false;
+    int chosen = -1;
+    for (size_t q = 0; q < p->cands.size(); q++)
+        if (p->cands[q]->variant == col[1]) chosen = int(q);
+    if (chosen < 0) return false;  // stale entry (kernel table changed)
+    std::stringstream fs(col[2]);
+    double f[8] = {0};
+    for (int x = 1; x < 8; x++) fs >> f[x];
+    std::vector<const KernelDesc *> fused;
+    if (col.size() > 3 && !col[3].empty()) {
+        std::stringstream ns(col[3]);
+        for (std::string n; std::getline(ns, n, ',');)
+            for (const KernelDesc *k : p->fused)
+                if (k->variant == n) fused.push_back(k);
+        if (fused.size() != p->fused.size()) return false;
+    }
+    p->chosen = chosen;
+    for (int x = 1; x < 8; x++) p->fcost[x] = f[x];
+    if (!fused.empty()) p->fused = fused;
+    return true;
+}
+
+static void tune_cache_store(const Plan *p) {
+    const char *path = std::getenv("SDAG_TUNE_CACHE");
+    if (!path || !*path) return;
+    std::lock_guard<std::mutex> lk(g_tune_file_mu);
+    std::ofstream out(path, std::ios::app);
+    if (!out) return;  // a cache is an optimisation: an unwritable path is not an error
+    out << tune_key(p) << "\t" << p->kernel().variant << "\t";
+    out.precision(17);
+    for (int x = 1; x < 8; x++) out << (x > 1 ? " " : "") << p->fcost[x];
+    out << "\t";
+    for (size_t q = 0; q < p->fused.size(); q++) out << (q ? "," : "") << p->fused[q]->variant;
+    out << "\n";
 }
 
 // Hierarchical autotuning, lite: time every candidate geometry on

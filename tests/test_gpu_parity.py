@@ -76,6 +76,31 @@ def test_tuned_plan_is_correct():
     check("lap25", dims, g, case)
 
 
+def test_persistent_tune_cache(tmp_path, monkeypatch):
+    """NEXT-3 persistent plan cache: a tune=1 plan appends its choice to
+    $SDAG_TUNE_CACHE; the next plan of the same shape restores it without timing."""
+    path = tmp_path / "tune.txt"
+    monkeypatch.setenv("SDAG_TUNE_CACHE", str(path))
+    dims = (40, 48, 64)
+    p1 = sdag.Plan(sdag.spec_text("smooth27"), dims, tune=True)
+    assert "[tuned]" in p1.describe()
+    lines = path.read_text().splitlines()
+    assert len(lines) == 1 and p1.info["variant"] in lines[0]
+    p2 = sdag.Plan(sdag.spec_text("smooth27"), dims, tune=True)
+    assert "from $SDAG_TUNE_CACHE" in p2.describe()
+    assert p2.info["variant"] == p1.info["variant"]
+    assert len(path.read_text().splitlines()) == 1
+    f1 = [ln for ln in p1.describe().splitlines() if "f(1)=" in ln]
+    f2 = [ln for ln in p2.describe().splitlines() if "f(1)=" in ln]
+    assert [x.split(":", 1)[1] for x in f1] == [x.split(":", 1)[1] for x in f2]
+    case = make_case("smooth27", dims)
+    g1, _ = run_gpu("smooth27", dims, case, variant=p1.info["variant"])
+    check("smooth27", dims, g1, case)
+    # another shape misses and appends
+    sdag.Plan(sdag.spec_text("smooth27"), (40, 48, 66), tune=True)
+    assert len(path.read_text().splitlines()) == 2
+
+
 def test_unaligned_pointer_uses_lsu_twin():
     dims = (12, 14, 16)
     case = make_case("jacobi7", dims)
