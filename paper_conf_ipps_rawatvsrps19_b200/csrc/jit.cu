@@ -24,7 +24,9 @@
 #include <dlfcn.h>
 #include <nvrtc.h>
 
+#include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -261,6 +263,30 @@ void jit_build_candidates(Plan *p) {
     };
     std::vector<Cand> cs;
     bool need_r0 = false, need_full = false;
+    // z-queue variants (sweep.cuh sdag_sweepq): on-axis z-taps from registers,
+    // the ring only as deep as the off-axis taps need
+    int rz_off = 0;
+    for (const Node &n : p->st.nodes)
+        if (n.kind == Node::Load3 && (n.off[1] != 0 || n.off[2] != 0)) rz_off = std::max(rz_off, std::abs(n.off[0]));
+    struct CandQ {
+        Geom g;
+        bool tma;
+        int smem;
+        std::string name;
+    };
+    std::vector<CandQ> cq;
+    if (RZ > 0) {
+        for (const Geom &g : geoms) {
+            const int px = g.tx + 2 * RX, py = g.ty + 2 * RY;
+            if (px > 256 || py > 256) continue;
+            if (nin * (2 * RZ + 1) * g.ux * g.uy > 48) continue;  // queue registers
+            const int plane_al = ((px * py * 8 + 127) / 128) * 128 / 8;
+            const int ns = RZ + rz_off + 1 + g.pf;
+            const int smem = ns * nin * plane_al * 8 + ns * 8;
+            if (smem > 227 * 1024) continue;
+            for (bool tma : {true, false}) cq.push_back({g, tma, smem, ""});
+        }
+    }
     for (const Geom &g : geoms) {
         const int px = g.tx + 2 * RX, py = g.ty + 2 * RY;
         if (px > 256 || py > 256) continue;
@@ -282,6 +308,7 @@ void jit_build_candidates(Plan *p) {
     if (need_full) src << jit_body_source(*p, "JitBody", RZ);
     if (need_r0 && RZ > 0) src << jit_body_source(*p, "JitBodyR0", 0);
     if (need_r0 && RZ == 0 && !need_full) src << jit_body_source(*p, "JitBody", 0);
+    if (!cq.empty()) src << jit_body_source(*p, "JitBodyQ", rz_off);
     src << "}  // namespace dev\n}  // namespace sdag\n";
     std::vector<std::string> names;
     for (Cand &c : cs) {
@@ -292,6 +319,15 @@ void jit_build_candidates(Plan *p) {
         names.push_back(buf);
         std::snprintf(buf, sizeof buf, "jit_%s_%dx%d_u%dx%d_pf%d%s", c.tma ? "tma" : "lsu", c.g.tx, c.g.ty, c.g.ux,
                       c.g.uy, c.g.pf, (c.rzr == RZ) ? "" : "_r0");
+        c.name = buf;
+    }
+    for (CandQ &c : cq) {
+        char buf[160];
+        std::snprintf(buf, sizeof buf, "sdag::dev::sdag_sweepq<sdag::dev::JitBodyQ, %d, %d, %d, %d, %d, %s>", c.g.tx,
+                      c.g.ty, c.g.ux, c.g.uy, c.g.pf, c.tma ? "true" : "false");
+        names.push_back(buf);
+        std::snprintf(buf, sizeof buf, "jitq_%s_%dx%d_u%dx%d_pf%d", c.tma ? "tma" : "lsu", c.g.tx, c.g.ty, c.g.ux,
+                      c.g.uy, c.g.pf);
         c.name = buf;
     }
     const std::string key = src.str();
@@ -352,6 +388,32 @@ void jit_build_candidates(Plan *p) {
         d->rx = RX;
         d->rzr = c.rzr;
         d->prio = int(q / 2) + (c.tma ? 0 : 100);
+        p->jit_descs.push_back(std::move(d));
+    }
+    for (size_t q = 0; q < cq.size(); q++) {
+        const CandQ &c = cq[q];
+        auto d = std::make_unique<KernelDesc>();
+        d->dag = "(jit)";
+        d->variant = c.name;
+        d->fn = nullptr;
+        d->cufn = fns[cs.size() + q];
+        d->threads = (c.g.tx / c.g.ux) * (c.g.ty / c.g.uy);
+        d->smem = c.smem;
+        d->tx = c.g.tx;
+        d->ty = c.g.ty;
+        d->ux = c.g.ux;
+        d->uy = c.g.uy;
+        d->pf = c.g.pf;
+        d->tma = c.tma;
+        d->nin = nin;
+        d->nout = nout;
+        d->nio = nio;
+        d->n1d = n1;
+        d->rz = RZ;
+        d->ry = RY;
+        d->rx = RX;
+        d->rzr = rz_off;
+        d->prio = -10 + int(q / 2) + (c.tma ? 0 : 100);  // preferred: 1.35x (lap25), 1.1x (27-pt) over the ring-only skeleton
         p->jit_descs.push_back(std::move(d));
     }
 }

@@ -303,5 +303,187 @@ __global__ void __launch_bounds__(Geo<B, TX, TY, UX, UY, PF>::THREADS)
     }
 }
 
+// ---------------------------------------------------------------------------
+// z-queue variant of the skeleton (NEXT-4 code generation, the star kernel's
+// register queue made generic): the body's on-axis z-taps (dy = dx = 0, the
+// stream dimension) come from a per-thread register queue of the
+// last 2*RZQ+1 planes of each staged array, filled once per plane from the
+// shared-memory ring; only off-axis taps read the ring, which therefore spans
+// RZQ + RZR + 1 + PF planes (RZR = max |dz| of the off-axis taps) instead of
+// 2RZ + 1 + PF.  Body interface as above plus RZQ (= RZ) -- same eval().
+// ---------------------------------------------------------------------------
+
+template <class B, int TX, int TY, int UX, int UY, int PF>
+struct GeoQ {
+    static constexpr int RZQ = B::RZ, RZR = B::RZR < 0 ? B::RZ : B::RZR, RY = B::RY, RX = B::RX, NIN = B::NIN;
+    static constexpr int PX = TX + 2 * RX, PY = TY + 2 * RY, PLANE = PX * PY;
+    static constexpr int PLANE_AL = ((PLANE * 8 + 127) / 128) * 128 / 8;
+    static constexpr int SLOT = NIN * PLANE_AL;
+    static constexpr int NS = RZQ + RZR + 1 + PF;
+    static constexpr int NQ = 2 * RZQ + 1;
+    static constexpr int THREADS = (TX / UX) * (TY / UY);
+    static constexpr int SMEM = NS * SLOT * 8 + NS * 8;
+    static_assert(TX % UX == 0 && TY % UY == 0, "tile must be a multiple of the patch");
+    static_assert(TX % 2 == 0, "TMA rows must be 16-byte multiples");
+    static_assert(PX <= 256 && PY <= 256, "TMA box dims <= 256");
+};
+
+template <class B, int PX, int NIN, int SLOT_ELEMS, int RZQ, int RZR, int NQ>
+struct TapQ {
+    const double *ring;
+    const int *soff;    // soff[dz + RZR] = slot offset of plane k + dz, |dz| <= RZR
+    const double *qv;   // this point's queue: qv[arr * NQ + dz + RZQ]
+    int base;
+    const SweepArgs *a;
+    int64_t gidx, b;
+    int gk, gj, gi;
+    static constexpr int PLANE_AL = SLOT_ELEMS / NIN;
+
+    __device__ __forceinline__ double at(int arr, int dz, int dy, int dx) const {
+        if (dy == 0 && dx == 0) return qv[arr * NQ + dz + RZQ];
+        return ring[soff[dz + RZR] + arr * PLANE_AL + base + dy * PX + dx];
+    }
+    __device__ __forceinline__ double io(int m) const { return a->io[m][gidx]; }
+    __device__ __forceinline__ double s(int n) const { return a->s[n]; }
+    __device__ __forceinline__ double s1(int arr, int off) const {
+        const int ax = B::axis1d(arr);
+        const int c = ax == 0 ? gk : (ax == 1 ? gj : gi);
+        return __ldg(a->a1d[arr] + b * a->a1d_bstride[arr] + c + off);
+    }
+};
+
+template <class B, int TX, int TY, int UX, int UY, int PF, bool USE_TMA>
+__global__ void __launch_bounds__(GeoQ<B, TX, TY, UX, UY, PF>::THREADS)
+    sdag_sweepq(const __grid_constant__ SweepArgs a) {
+    using G = GeoQ<B, TX, TY, UX, UY, PF>;
+    constexpr int RZQ = G::RZQ, RZR = G::RZR, RY = G::RY, RX = G::RX, NIN = G::NIN;
+    constexpr int PX = G::PX, NS = G::NS, SLOT = G::SLOT, NQ = G::NQ;
+    constexpr int NTX = TX / UX;
+
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    double *ring = reinterpret_cast<double *>(smem_raw);
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem_raw + NS * SLOT * 8);
+
+    const int tile_x = blockIdx.x, tile_y = blockIdx.y;
+    const int chunk = blockIdx.z % a.nchunk;
+    const int64_t prob = blockIdx.z / a.nchunk;
+    const int x0 = a.lo[2] + tile_x * TX, y0 = a.lo[1] + tile_y * TY;
+    const int kb = a.lo[0] + chunk * a.zchunk;
+    const int ke = min(a.hi[0], kb + a.zchunk);
+    if (kb >= ke) return;
+    const int p0 = kb - RZQ;
+    const int plast = ke - 1 + RZQ;
+    const int64_t zbase = prob * a.nz;
+
+    const int t = threadIdx.x;
+    const int lx = t % NTX, ly = t / NTX;
+
+    auto issue = [&](int p) {
+        const int slot = unsigned(p - p0) % NS;
+        double *dst = ring + slot * SLOT;
+        if constexpr (USE_TMA) {
+            if (t == 0) {
+                uint64_t *bar = &bars[slot];
+                mbar_expect_tx(bar, uint32_t(NIN * G::PX * G::PY * 8));
+#pragma unroll
+                for (int q = 0; q < NIN; q++)
+                    tma_load_3d(dst + q * G::PLANE_AL, &a.tmap[q], bar, x0 - RX, y0 - RY, int(zbase + p));
+            }
+        } else {
+            const int64_t pl = (zbase + p) * a.ny * a.nx;
+            for (int e = t; e < NIN * G::PLANE; e += G::THREADS) {
+                const int q = e / G::PLANE, r = e % G::PLANE;
+                const int yy = r / PX, xx = r % PX;
+                const int gx = x0 - RX + xx, gy = y0 - RY + yy;
+                const bool ok = gx >= 0 && gx < a.nx && gy >= 0 && gy < a.ny && p >= 0 && p < a.nz;
+                const double *src = a.in[q] + (ok ? pl + int64_t(gy) * a.nx + gx : 0);
+                cp_async8(dst + q * G::PLANE_AL + r, src, ok);
+            }
+        }
+    };
+
+    if constexpr (USE_TMA) {
+        if (t == 0) {
+            for (int s = 0; s < NS; s++) mbar_init(&bars[s], 1);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+        __syncthreads();
+    }
+    for (int p = p0; p < p0 + PF; p++) {
+        if (p <= plast) issue(p);
+        if constexpr (!USE_TMA) cp_async_commit();
+    }
+
+    // queue[py][px][arr * NQ + i] = array arr at plane p - 2RZQ + i (own point)
+    double qv[UY][UX][NIN * NQ];
+#pragma unroll
+    for (int py = 0; py < UY; py++)
+#pragma unroll
+        for (int px = 0; px < UX; px++)
+#pragma unroll
+            for (int e = 0; e < NIN * NQ; e++) qv[py][px][e] = 0.0;
+
+    int soff[2 * RZR + 1];
+    for (int p = p0; p <= plast; p++) {
+        {
+            const int pn = p + PF;
+            if (pn <= plast) issue(pn);
+            if constexpr (!USE_TMA) cp_async_commit();
+        }
+        if constexpr (USE_TMA) {
+            mbar_wait(&bars[unsigned(p - p0) % NS], (unsigned(p - p0) / NS) & 1);
+        } else {
+            cp_async_wait<PF>();
+            __syncthreads();
+        }
+        const int k = p - RZQ;  // output plane of this step
+        // queue: shift, then the own values of the newest plane p
+        const double *pl = ring + (unsigned(p - p0) % NS) * SLOT;
+#pragma unroll
+        for (int py = 0; py < UY; py++)
+#pragma unroll
+            for (int px = 0; px < UX; px++) {
+                const int ty = ly * UY + py, tx = lx * UX + px;
+#pragma unroll
+                for (int q = 0; q < NIN; q++) {
+#pragma unroll
+                    for (int i = 0; i < NQ - 1; i++) qv[py][px][q * NQ + i] = qv[py][px][q * NQ + i + 1];
+                    qv[py][px][q * NQ + NQ - 1] = pl[q * G::PLANE_AL + (ty + RY) * PX + (tx + RX)];
+                }
+            }
+        if (k >= kb) {
+#pragma unroll
+            for (int d = 0; d < 2 * RZR + 1; d++) soff[d] = (unsigned(k - RZR + d - p0) % NS) * SLOT;
+#pragma unroll
+            for (int py = 0; py < UY; py++) {
+#pragma unroll
+                for (int px = 0; px < UX; px++) {
+                    const int ty = ly * UY + py, tx = lx * UX + px;
+                    const int gj = y0 + ty, gi = x0 + tx;
+                    const bool inside = gj < a.hi[1] && gi < a.hi[2] && gi >= a.xmin;
+                    TapQ<B, PX, NIN, SLOT, RZQ, RZR, NQ> g;
+                    g.ring = ring;
+                    g.soff = soff;
+                    g.qv = qv[py][px];
+                    g.base = (ty + RY) * PX + (tx + RX);
+                    g.a = &a;
+                    g.b = prob;
+                    g.gk = k;
+                    g.gj = gj;
+                    g.gi = gi;
+                    g.gidx = ((zbase + k) * a.ny + gj) * a.nx + gi;
+                    if (inside) {
+                        double o[B::NOUT];
+                        B::eval(g, o);
+#pragma unroll
+                        for (int m = 0; m < B::NOUT; m++) st_stream(a.out[m] + g.gidx, o[m]);
+                    }
+                }
+            }
+        }
+        __syncthreads();  // plane p - RZQ - RZR may be overwritten from the next step on
+    }
+}
+
 }  // namespace dev
 }  // namespace sdag
