@@ -4,7 +4,9 @@
 #include "kdesc.cuh"
 namespace sdag {
 void add_kernels_hypterm(std::vector<KernelDesc> &v) {
-    SDAG_HYP_PAIR(v, "hypterm", 64, 8, 2, 0);  // 0.796 ms at 320^3 (pf1: 0.826)
+    SDAG_HYP_PAIR(v, "hypterm", 64, 8, 2, 0);  // 0.793-0.796 ms at 320^3 (pf1: 0.826)
+    // cropped per-array boxes: 0.799 ms (32x16: 0.874), no gain -- DESIGN 6.4
+    SDAG_HYPC_PAIR(v, "hypterm", 64, 8, 2, 1);
     SDAG_HYP_PAIR(v, "hypterm", 16, 16, 2, 1);
     SDAG_HYP_PAIR(v, "hypterm", 64, 8, 1, 2);
     SDAG_HYP_PAIR(v, "hypterm", 32, 16, 1, 3);

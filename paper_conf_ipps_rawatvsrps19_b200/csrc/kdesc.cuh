@@ -146,6 +146,41 @@ KernelDesc make_hyp_desc(const char *dag, int prio) {
     return d;
 }
 
+// hypterm with cropped per-array boxes (hyp.cuh, sdag_hypc)
+template <int TX, int TY, int PF, bool TMA>
+KernelDesc make_hypc_desc(const char *dag, int prio) {
+    using G = dev::HypcGeo<TX, TY, PF>;
+    KernelDesc d;
+    d.dag = dag;
+    d.tx = TX;
+    d.ty = TY;
+    d.ux = 2;
+    d.uy = 1;
+    d.pf = PF;
+    d.tma = TMA;
+    d.nin = 8;
+    d.nout = 5;
+    d.rz = 4;
+    d.ry = 4;
+    d.rx = 4;
+    d.rzr = 4;  // z-halo planes streamed per chunk
+    d.prio = prio;
+    char buf[96];
+    std::snprintf(buf, sizeof buf, "hypc_%s_%dx%d_u2x1_pf%d", TMA ? "tma" : "lsu", TX, TY, PF);
+    d.variant = buf;
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_hypc<TX, TY, PF, TMA>);
+    d.threads = G::THREADS;
+    d.smem = G::SMEM;
+    for (int q = 0; q < G::NA; q++) d.inbox.emplace_back(G::px(q), G::py(q));
+    return d;
+}
+
+#define SDAG_HYPC_PAIR(v, DAG, TX, TY, PF, PRIO)                                  \
+    do {                                                                          \
+        v.push_back(make_hypc_desc<TX, TY, PF, true>(DAG, PRIO));                 \
+        v.push_back(make_hypc_desc<TX, TY, PF, false>(DAG, PRIO + 100));          \
+    } while (0)
+
 #define SDAG_HYP_PAIR(v, DAG, TX, TY, PF, PRIO)                                   \
     do {                                                                          \
         v.push_back(make_hyp_desc<TX, TY, PF, true>(DAG, PRIO));                  \

@@ -2,6 +2,7 @@
 #pragma once
 
 #include <string>
+#include <utility>
 #include <vector>
 
 namespace sdag {
@@ -20,6 +21,7 @@ struct KernelDesc {
     int prio = 0;                         // heuristic preference (lower first)
     int tsteps = 1;                       // sweeps fused per launch (temporal fusion, NEXT-1)
     double fhint = 0.0;                   // measured f(x): launch cost / one sweep (0 = generic estimate)
+    std::vector<std::pair<int, int>> inbox;  // per staged input: TMA box (x, y) if cropped (else tx+2rx, ty+2ry)
     void *cufn = nullptr;                 // CUfunction of an NVRTC-compiled kernel (jit.cu); fn is then null
 };
 

@@ -227,7 +227,12 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *
         const Formal &fo = p->st.formal(ArgKind::Array3D, f);
         if (p->in_slot[f] >= 0) {
             A.in[p->in_slot[f]] = a3[f];
-            if (k.tma) A.tmap[p->in_slot[f]] = tmap_for(p, a3[f], dims[2], dims[1], nzt, k.tx + 2 * k.rx, k.ty + 2 * k.ry);
+            if (k.tma) {
+                const int s = p->in_slot[f];
+                const bool crop = s < int(k.inbox.size());
+                A.tmap[s] = tmap_for(p, a3[f], dims[2], dims[1], nzt, crop ? k.inbox[s].first : k.tx + 2 * k.rx,
+                                     crop ? k.inbox[s].second : k.ty + 2 * k.ry);
+            }
         }
         if (p->out_slot[f] >= 0) A.out[p->out_slot[f]] = a3[f];
         if (p->io_slot[f] >= 0) A.io[p->io_slot[f]] = a3[f];
