@@ -294,6 +294,48 @@ sdag_status sdag_dist_apply_iterated_loopback(sdag_dist *dists, int32_t nranks, 
                                               double *const *buf1, int32_t T, const double *scalars,
                                               int32_t nscalars, sdag_stream stream);
 
+/* Peer-memory halo path for iterated slabs ("B200-native
+ * alternative"; NEXT-4).  Instead of an NCCL send/recv step, the sweep kernel
+ * that computes a slab's boundary planes stores each of them twice: into its
+ * own output and, over NVLink P2P, into the ghost planes of the neighbour that
+ * reads them next sweep (store-side fusion, tile by tile).  The ordering is a
+ * 32-bit flag word per neighbour in each rank's HBM, written by the neighbour
+ * with a system-scope release after its boundary launch and waited on (acquire)
+ * by this rank's stream before the launch that reads the ghosts.
+ *
+ * Usage (every rank, same spec/dims/opts/T; opts.tune = 0 so all ranks derive
+ * the same launch schedule):
+ *   sdag_dist_create(..., rank, nranks, NULL, &d);   (no NCCL communicator)
+ *   sdag_dist_p2p_alloc(d, &buf0, &buf1);
+ *   exchange handles: sdag_dist_p2p_handle(d, h) -> all-gather on the host ->
+ *   sdag_dist_p2p_attach(d, 0, h_of(rank-1)), sdag_dist_p2p_attach(d, 1, h_of(rank+1))
+ *   (or sdag_dist_p2p_attach_local(d, side, peer) for slabs of one process);
+ *   fill buf0 (layout of sdag_dist_layout), then
+ *   sdag_dist_p2p_apply_iterated(d, T, scalars, n, stream)  -> result in buf[T&1].
+ *
+ * sdag_dist_p2p_alloc: the library allocates ONE device region holding buf0,
+ *   buf1 (each nz_alloc*ny*nx doubles, C order, 4 KiB-aligned) and the flag
+ *   words, zero-filled; it is owned by the dist (freed by sdag_dist_destroy).
+ *   Repeated calls return the same buffers.
+ * sdag_dist_p2p_handle: the cudaIpcMemHandle_t (64 bytes) of that region.
+ * sdag_dist_p2p_attach: side 0 = rank-1, 1 = rank+1; opens the neighbour's
+ *   handle (another process; cudaIpcOpenMemHandle with lazy peer access).
+ *   INVALID_ARG if there is no neighbour on that side or alloc was not called.
+ * sdag_dist_p2p_attach_local: same for a neighbour dist of this process
+ *   (its region is used directly; peer access is enabled if on another device).
+ * sdag_dist_p2p_apply_iterated: T sweeps of a 1-in/1-out plan over buf0/buf1
+ *   (fused launches as sdag_dist_apply_iterated), enqueued on `stream` only;
+ *   bit-identical to the single-GPU schedule.  Consecutive calls on a rank are
+ *   ordered against the neighbours' previous calls by the same flags.  A wait
+ *   that does not complete within SDAG_P2P_TIMEOUT_S seconds (default 60)
+ *   traps the kernel (the error surfaces at the next synchronisation). */
+sdag_status sdag_dist_p2p_alloc(sdag_dist d, double **buf0, double **buf1);
+sdag_status sdag_dist_p2p_handle(sdag_dist d, uint8_t handle[64]);
+sdag_status sdag_dist_p2p_attach(sdag_dist d, int32_t side, const uint8_t handle[64]);
+sdag_status sdag_dist_p2p_attach_local(sdag_dist d, int32_t side, sdag_dist peer);
+sdag_status sdag_dist_p2p_apply_iterated(sdag_dist d, int32_t T, const double *scalars, int32_t nscalars,
+                                         sdag_stream stream);
+
 /* ------------------------------------------------------------------------
  * Diagnostics
  * ------------------------------------------------------------------------ */

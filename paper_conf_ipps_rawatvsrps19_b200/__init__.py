@@ -396,6 +396,46 @@ class Dist:
                                                             _stream_handle(stream)))
 
 
+    # ---- peer-memory halo path (NVLink P2P stores from the sweep kernels) ----
+    def p2p_alloc(self):
+        """(buf0, buf1): the library-owned slab buffers of sdag_dist_p2p_alloc as
+        float64 CUDA tensors of the local layout (views; valid while this dist lives)"""
+        import torch
+        b0, b1 = ctypes.c_void_p(), ctypes.c_void_p()
+        _check(self._L.sdag_dist_p2p_alloc(self._h, ctypes.byref(b0), ctypes.byref(b1)))
+        shape = tuple(int(x) for x in self.layout()[0])
+        dev = torch.device("cuda", torch.cuda.current_device())
+        return tuple(torch.as_tensor(_DeviceView(b.value, shape), device=dev) for b in (b0, b1))
+
+    def p2p_handle(self) -> bytes:
+        h = ctypes.create_string_buffer(64)
+        _check(self._L.sdag_dist_p2p_handle(self._h, h))
+        return h.raw
+
+    def p2p_attach(self, side, handle):
+        """side 0 = rank-1, 1 = rank+1; `handle` from that rank's p2p_handle()
+        (another process), or a Dist of this process"""
+        if isinstance(handle, Dist):
+            _check(self._L.sdag_dist_p2p_attach_local(self._h, int(side), handle._h))
+        else:
+            if len(handle) != 64:
+                raise ValueError("an IPC handle is 64 bytes")
+            _check(self._L.sdag_dist_p2p_attach(self._h, int(side), bytes(handle)))
+
+    def p2p_apply_iterated(self, T, scalars=(), stream=None):
+        """T sweeps over the p2p buffers; result in buf[T & 1]"""
+        s, ns = _scal(scalars)
+        _check(self._L.sdag_dist_p2p_apply_iterated(self._h, int(T), s, ns, _stream_handle(stream)))
+
+
+class _DeviceView:
+    """__cuda_array_interface__ of a float64 C-order device buffer (zero copy)"""
+
+    def __init__(self, ptr, shape):
+        self.__cuda_array_interface__ = {"shape": shape, "typestr": "<f8", "data": (int(ptr), False),
+                                         "version": 3, "strides": None}
+
+
 def launch_count() -> int:
     return int(_capi.lib().sdag_launch_count())
 

@@ -89,6 +89,11 @@ def lib():
             "sdag_dist_apply_iterated_loopback": (S, [ctypes.POINTER(P), c_i32, ctypes.POINTER(c_void_p),
                                                       ctypes.POINTER(c_void_p), c_i32, c_dblp, c_i32, P]),
             "sdag_dist_destroy": (None, [P]),
+            "sdag_dist_p2p_alloc": (S, [P, ctypes.POINTER(c_void_p), ctypes.POINTER(c_void_p)]),
+            "sdag_dist_p2p_handle": (S, [P, ctypes.c_char_p]),
+            "sdag_dist_p2p_attach": (S, [P, c_i32, ctypes.c_char_p]),
+            "sdag_dist_p2p_attach_local": (S, [P, c_i32, P]),
+            "sdag_dist_p2p_apply_iterated": (S, [P, c_i32, c_dblp, c_i32, P]),
             "sdag_last_error": (c_char_p, []),
             "sdag_version": (c_char_p, []),
             "sdag_launch_count": (c_i64, []),
@@ -113,6 +118,8 @@ EXPORTED = [
     "sdag_apply_host", "sdag_fusion_schedule", "sdag_slab_partition", "sdag_slab_halo",
     "sdag_slab_partition2", "sdag_slab_halo2", "sdag_nccl_get_unique_id", "sdag_nccl_comm_create",
     "sdag_nccl_comm_destroy", "sdag_dist_create", "sdag_dist_layout", "sdag_dist_local_plan", "sdag_dist_apply",
-    "sdag_dist_apply_iterated", "sdag_dist_destroy", "sdag_dist_apply_iterated_loopback", "sdag_last_error",
+    "sdag_dist_apply_iterated", "sdag_dist_destroy", "sdag_dist_apply_iterated_loopback",
+    "sdag_dist_p2p_alloc", "sdag_dist_p2p_handle", "sdag_dist_p2p_attach", "sdag_dist_p2p_attach_local",
+    "sdag_dist_p2p_apply_iterated", "sdag_last_error",
     "sdag_version", "sdag_launch_count", "sdag_measure_fp64_peak", "sdag_registry_count", "sdag_registry_get",
 ]

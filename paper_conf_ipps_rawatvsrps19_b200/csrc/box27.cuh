@@ -46,7 +46,7 @@ struct BoxGeo {
 //   retimed form: T_k = s1_k - 6 s0_k + s0_{k-1} is formed when plane k
 //   streams past and B[k] = a A[k] - (b h2inv)(T_k + s0_{k+1}) when plane k+1
 //   does (2 doubles of z-state per point).
-template <int TX, int TY, int UY, int PF, bool USE_TMA, int FORM = 0>
+template <int TX, int TY, int UY, int PF, bool USE_TMA, int FORM = 0, bool MIR = false>
 __global__ void __launch_bounds__(BoxGeo<TX, TY, UY, PF>::THREADS)
     sdag_box27(const __grid_constant__ SweepArgs a) {
     using G = BoxGeo<TX, TY, UY, PF>;
@@ -155,6 +155,7 @@ __global__ void __launch_bounds__(BoxGeo<TX, TY, UY, PF>::THREADS)
         }
         const int k = p - 1;  // output plane finished by this plane
         double *o = a.out[0] + ((zbase + k) * a.ny + (y0 + cy)) * a.nx + gi;
+        const bool mp = MIR && mirror_plane(a, k);
 #pragma unroll
         for (int py = 0; py < UY; py++) {
             double res[2];
@@ -179,9 +180,12 @@ __global__ void __launch_bounds__(BoxGeo<TX, TY, UY, PF>::THREADS)
             if (k >= kb && py < nrows) {
                 if (vec) {
                     __stcs(reinterpret_cast<double2 *>(o), make_double2(res[0], res[1]));
+                    if constexpr (MIR) if (mp) mirror2(a, k, o, res[0], res[1]);
                 } else {
                     if (ok0) __stcs(o, res[0]);
                     if (ok1) __stcs(o + 1, res[1]);
+                    if (MIR && mp && ok0) mirror1(a, k, o, res[0]);
+                    if (MIR && mp && ok1) mirror1(a, k, o + 1, res[1]);
                 }
             }
             o += a.nx;

@@ -328,6 +328,38 @@ sdag_status sdag_dist_apply_iterated_loopback(sdag_dist *dists, int32_t nranks, 
 
 void sdag_dist_destroy(sdag_dist d) { delete reinterpret_cast<sdag::Dist *>(d); }
 
+sdag_status sdag_dist_p2p_alloc(sdag_dist d, double **buf0, double **buf1) {
+    return guard([&] { sdag::dist_p2p_alloc(reinterpret_cast<sdag::Dist *>(d), buf0, buf1); });
+}
+
+sdag_status sdag_dist_p2p_handle(sdag_dist d, uint8_t handle[64]) {
+    return guard([&] {
+        if (!handle) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null handle");
+        sdag::dist_p2p_handle(reinterpret_cast<sdag::Dist *>(d), handle);
+    });
+}
+
+sdag_status sdag_dist_p2p_attach(sdag_dist d, int32_t side, const uint8_t handle[64]) {
+    return guard([&] {
+        if (!d || !handle) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null argument");
+        sdag::dist_p2p_attach(reinterpret_cast<sdag::Dist *>(d), side, handle);
+    });
+}
+
+sdag_status sdag_dist_p2p_attach_local(sdag_dist d, int32_t side, sdag_dist peer) {
+    return guard([&] {
+        if (side != 0 && side != 1) throw sdag::Error(SDAG_ERR_INVALID_ARG, "side must be 0 or 1");
+        sdag::dist_p2p_attach_local(reinterpret_cast<sdag::Dist *>(d), side, reinterpret_cast<sdag::Dist *>(peer));
+    });
+}
+
+sdag_status sdag_dist_p2p_apply_iterated(sdag_dist d, int32_t T, const double *s, int32_t ns, sdag_stream stream) {
+    return guard([&] {
+        sdag::dist_p2p_apply_iterated(reinterpret_cast<sdag::Dist *>(d), T, s, ns,
+                                      reinterpret_cast<cudaStream_t>(stream));
+    });
+}
+
 // ---- diagnostics ------------------------------------------------------------
 
 const char *sdag_last_error(void) { return g_err.c_str(); }

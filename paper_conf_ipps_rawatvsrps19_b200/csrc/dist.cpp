@@ -158,6 +158,9 @@ void nccl_comm_destroy(void *c) {
 // ---------------------------------------------------------------------------
 
 Dist::~Dist() {
+    for (void *m : peer_ipc)
+        if (m) cudaIpcCloseMemHandle(m);
+    if (p2p_base) cudaFree(p2p_base);
     if (own_comm) cudaStreamDestroy(own_comm);
     if (ev_ready) cudaEventDestroy(ev_ready);
     if (ev_halo) cudaEventDestroy(ev_halo);
@@ -420,6 +423,197 @@ void dist_apply_iterated_loopback(Dist **ds, int n, double *const *b0, double *c
             a3[fout] = out(r);
             sweep_split(ds[r], k0 ? *k0 : single_kernel(ds[r]->local, in(r)), a3, nullptr, s, stream, stream, false);
         }
+        t++;
+    }
+}
+
+
+
+// ---------------------------------------------------------------------------
+// peer-memory halo path (p2p)
+//
+// Launch t of a call reads buf[t&1] (input) and writes buf[(t+1)&1].  Its
+// boundary bands -- owned planes [H, 2H) and [nz_own, nz_own + H), the planes
+// the neighbours hold as ghosts -- are stored by the sweep kernel itself both
+// locally and into the neighbour's buf[(t+1)&1] ghost planes (Mirror), after
+// this rank's stream has waited for the neighbours' flag >= e_t = base + t:
+//  * the neighbour finished launch t-1, so its stores into MY buf[t&1] ghosts
+//    (read now) have landed, and
+//  * it finished reading ITS buf[(t+1)&1] (= its input of launch t-1), into
+//    whose ghosts these stores go.
+// After the boundary launch the rank signals e_t + 1.  The interior planes
+// [2H, nz_own) read and write no ghost plane: they run first, with no wait.
+// Before launch 0 the input bands of buf0 are pushed (cudaMemcpyAsync over
+// P2P) after the neighbours' previous call ended, and `base` is signalled.
+// Kernels without a KernelDesc::fn_mirror instantiation push their output
+// bands the same way.
+// ---------------------------------------------------------------------------
+
+namespace {
+
+size_t p2p_buf_bytes(int64_t nz_alloc, int64_t ny, int64_t nx) {
+    const size_t b = size_t(nz_alloc) * size_t(ny) * size_t(nx) * 8;
+    return (b + 4095) / 4096 * 4096;
+}
+
+void p2p_map_peer(Dist *d, int side, void *base) {
+    if (side != 0 && side != 1) throw Error(SDAG_ERR_INVALID_ARG, "side must be 0 (lower) or 1 (upper)");
+    const int nr = d->rank + (side == 0 ? -1 : 1);
+    if (nr < 0 || nr >= d->nranks) throw Error(SDAG_ERR_INVALID_ARG, "no neighbour on that side");
+    const Slab ns = slab_partition(d->gnz, d->rz, d->nranks, nr, d->time_tile);
+    const size_t bb = p2p_buf_bytes(ns.nz_alloc, d->local->dims[1], d->local->dims[2]);
+    char *b = static_cast<char *>(base);
+    d->peer_buf[side][0] = reinterpret_cast<double *>(b);
+    d->peer_buf[side][1] = reinterpret_cast<double *>(b + bb);
+    uint32_t *pf = reinterpret_cast<uint32_t *>(b + 2 * bb);
+    d->peer_flag[side] = pf + (side == 0 ? 1 : 0);  // I am my lower neighbour's upper side
+    // global g = z0 - H + k (mine) = z0' - H + k' (neighbour's)
+    d->peer_shift[side] = d->slab.z0 - ns.z0;
+}
+
+}  // namespace
+
+void dist_p2p_alloc(Dist *d, double **buf0, double **buf1) {
+    if (!d) throw Error(SDAG_ERR_INVALID_ARG, "null dist");
+    if (d->local->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
+    check_cuda(cudaSetDevice(d->local->device), "cudaSetDevice");
+    if (!d->p2p_base) {
+        const int64_t *dims = d->local->dims;
+        d->p2p_buf_bytes = p2p_buf_bytes(dims[0], dims[1], dims[2]);
+        const size_t total = 2 * d->p2p_buf_bytes + 4096;
+        check_cuda(cudaMalloc(&d->p2p_base, total), "cudaMalloc(p2p slab buffers)");
+        char *b = static_cast<char *>(d->p2p_base);
+        d->p2p_buf[0] = reinterpret_cast<double *>(b);
+        d->p2p_buf[1] = reinterpret_cast<double *>(b + d->p2p_buf_bytes);
+        d->p2p_flags = reinterpret_cast<uint32_t *>(b + 2 * d->p2p_buf_bytes);
+        check_cuda(cudaMemset(d->p2p_base, 0, total), "cudaMemset(p2p)");
+        check_cuda(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
+        d->epoch = 0;
+    }
+    if (buf0) *buf0 = d->p2p_buf[0];
+    if (buf1) *buf1 = d->p2p_buf[1];
+}
+
+void dist_p2p_handle(Dist *d, uint8_t handle[64]) {
+    if (!d || !d->p2p_base) throw Error(SDAG_ERR_INVALID_ARG, "call sdag_dist_p2p_alloc first");
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+    cudaIpcMemHandle_t h;
+    check_cuda(cudaIpcGetMemHandle(&h, d->p2p_base), "cudaIpcGetMemHandle");
+    std::memcpy(handle, &h, 64);
+}
+
+void dist_p2p_attach(Dist *d, int side, const uint8_t handle[64]) {
+    if (!d || !d->p2p_base) throw Error(SDAG_ERR_INVALID_ARG, "call sdag_dist_p2p_alloc first");
+    if (side != 0 && side != 1) throw Error(SDAG_ERR_INVALID_ARG, "side must be 0 (lower) or 1 (upper)");
+    check_cuda(cudaSetDevice(d->local->device), "cudaSetDevice");
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, handle, 64);
+    void *m = nullptr;
+    check_cuda(cudaIpcOpenMemHandle(&m, h, cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle");
+    if (d->peer_ipc[side]) cudaIpcCloseMemHandle(d->peer_ipc[side]);
+    d->peer_ipc[side] = m;
+    p2p_map_peer(d, side, m);
+}
+
+void dist_p2p_attach_local(Dist *d, int side, Dist *peer) {
+    if (!d || !d->p2p_base || !peer || !peer->p2p_base)
+        throw Error(SDAG_ERR_INVALID_ARG, "both dists need sdag_dist_p2p_alloc first");
+    if (peer->nranks != d->nranks || peer->rank != d->rank + (side == 0 ? -1 : 1))
+        throw Error(SDAG_ERR_INVALID_ARG, "peer is not this rank's neighbour on that side");
+    if (peer->local->device != d->local->device) {
+        int ok = 0;
+        check_cuda(cudaDeviceCanAccessPeer(&ok, d->local->device, peer->local->device), "cudaDeviceCanAccessPeer");
+        if (!ok) throw Error(SDAG_ERR_DEVICE, "devices cannot access each other's memory");
+        check_cuda(cudaSetDevice(d->local->device), "cudaSetDevice");
+        const cudaError_t e = cudaDeviceEnablePeerAccess(peer->local->device, 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) check_cuda(e, "cudaDeviceEnablePeerAccess");
+        cudaGetLastError();
+    }
+    p2p_map_peer(d, side, peer->p2p_base);
+}
+
+void dist_p2p_apply_iterated(Dist *d, int T, const double *s, int ns, cudaStream_t st) {
+    if (!d || !d->p2p_base) throw Error(SDAG_ERR_INVALID_ARG, "call sdag_dist_p2p_alloc first");
+    Plan *p = d->local;
+    if (p->n3() != 2 || p->an.n_in != 1 || p->an.n_out != 1 || p->n1() != 0)
+        throw Error(SDAG_ERR_INVALID_ARG, "iterated dist apply needs a 1-input 1-output plan");
+    if (ns != p->ns() || T < 0) throw Error(SDAG_ERR_INVALID_ARG, "bad arguments");
+    const Slab &S = d->slab;
+    const int has[2] = {S.has_lower, S.has_upper};
+    for (int q = 0; q < 2; q++)
+        if (has[q] && !d->peer_buf[q][0])
+            throw Error(SDAG_ERR_INVALID_ARG, std::string("no ") + (q ? "upper" : "lower") +
+                                                  " neighbour attached (sdag_dist_p2p_attach)");
+    int fin = -1, fout = -1;
+    for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
+    check_cuda(cudaSetDevice(p->device), "cudaSetDevice");
+    if (T == 0) return;
+
+    const int64_t H = S.halo;
+    const size_t plane = size_t(p->dims[1] * p->dims[2]);
+    const size_t band = size_t(H) * plane * 8;
+    double **buf = d->p2p_buf;
+    // bands, in my local planes: [H, 2H) goes to the lower neighbour, [nz_own, nz_own+H) to the upper
+    const int64_t band_lo[2] = {H, S.nz_own};
+    auto push = [&](int b) {  // my bands of buffer b -> the neighbours' ghost planes of their buffer b
+        for (int q = 0; q < 2; q++)
+            if (has[q])
+                check_cuda(cudaMemcpyAsync(d->peer_buf[q][b] + size_t(band_lo[q] + d->peer_shift[q]) * plane,
+                                           buf[b] + size_t(band_lo[q]) * plane, band, cudaMemcpyDefault, st),
+                           "p2p band push");
+    };
+    auto signal = [&](uint32_t v) {
+        p2p_signal(has[0] ? d->peer_flag[0] : nullptr, has[1] ? d->peer_flag[1] : nullptr, v, st);
+        d->epoch = v;
+    };
+    auto wait = [&](uint32_t v) {
+        const uint32_t need[2] = {v, v};
+        p2p_wait(d->p2p_flags, need, has, st);
+    };
+
+    // every kernel this call launches is loaded before the first flag wait is
+    // enqueued (lazy loading of a kernel can block behind a spinning wait)
+    const std::vector<const KernelDesc *> sched = iter_schedule(d, buf[0], buf[1], T);
+    p2p_preload();
+    for (const KernelDesc *k0 : sched) {
+        const KernelDesc &k = k0 ? *k0 : single_kernel(p, buf[0]);
+        cudaFuncAttributes fa;
+        for (const void *fn : {k.fn, k.fn_mirror})
+            if (fn) check_cuda(cudaFuncGetAttributes(&fa, fn), "cudaFuncGetAttributes");
+    }
+
+    wait(d->epoch);  // the neighbours' previous call is over (first call: 0)
+    push(0);
+    const uint32_t base = d->epoch + 1;
+    signal(base);
+
+    int64_t zr[2];
+    global_interior(d, zr);
+    const Ranges r = ranges_of(d, H);  // bands of full ghost depth: every plane a neighbour reads
+    int cur = 0;
+    uint32_t t = 0;
+    for (const KernelDesc *k0 : sched) {
+        const KernelDesc &k = k0 ? *k0 : single_kernel(p, buf[cur]);
+        double *a3[2];
+        a3[fin] = buf[cur];
+        a3[fout] = buf[1 - cur];
+        if (r.split && r.in_hi > r.in_lo) plan_launch(p, k, a3, nullptr, s, 1, r.in_lo, r.in_hi, st, nullptr, zr);
+        wait(base + t);
+        Mirror m;
+        if (k.fn_mirror)
+            for (int q = 0; q < 2; q++)
+                if (has[q]) {
+                    m.peer[q] = d->peer_buf[q][1 - cur];
+                    m.off[q] = d->peer_shift[q] * int64_t(plane);
+                    m.klo[q] = int32_t(band_lo[q]);
+                    m.khi[q] = int32_t(band_lo[q] + H);
+                }
+        for (int q = 0; q < 2; q++)
+            if (r.b_hi[q] > r.b_lo[q])
+                plan_launch(p, k, a3, nullptr, s, 1, r.b_lo[q], r.b_hi[q], st, nullptr, zr, k.fn_mirror ? &m : nullptr);
+        if (!k.fn_mirror) push(1 - cur);
+        signal(base + t + 1);
+        cur = 1 - cur;
         t++;
     }
 }

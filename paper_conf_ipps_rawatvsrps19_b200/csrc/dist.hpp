@@ -41,6 +41,17 @@ struct Dist {
     void *comm = nullptr;   // ncclComm_t (not owned)
     cudaStream_t own_comm = nullptr;
     cudaEvent_t ev_ready = nullptr, ev_halo = nullptr;
+    // peer-memory halo path (p2p): one allocation buf0 | buf1 | flags owned here,
+    // the neighbours' allocations mapped (CUDA IPC, or same-process pointers)
+    void *p2p_base = nullptr;
+    size_t p2p_buf_bytes = 0;
+    double *p2p_buf[2] = {nullptr, nullptr};
+    uint32_t *p2p_flags = nullptr;        // [0] written by the lower neighbour, [1] by the upper
+    double *peer_buf[2][2] = {};          // [side][buffer] of the neighbours (0 lower, 1 upper)
+    uint32_t *peer_flag[2] = {};          // the neighbour's word this rank writes
+    int64_t peer_shift[2] = {0, 0};       // my local plane k is the neighbour's plane k + shift
+    void *peer_ipc[2] = {};               // opened IPC mappings (closed in ~Dist)
+    uint32_t epoch = 0;                   // last flag value this rank signalled
     ~Dist();
 };
 
@@ -52,6 +63,15 @@ void dist_apply_iterated(Dist *d, double *b0, double *b1, int T, const double *s
                          cudaStream_t comm);
 void dist_apply_iterated_loopback(Dist **d, int n, double *const *b0, double *const *b1, int T, const double *s,
                                   int ns, cudaStream_t stream);
+
+// peer-memory halo path (SURVEY 8(e) B200-native alternative): the launches
+// that compute a slab's boundary planes also store them into the neighbours'
+// ghost planes (NVLink P2P), ordered by per-neighbour flag words; no NCCL.
+void dist_p2p_alloc(Dist *d, double **buf0, double **buf1);
+void dist_p2p_handle(Dist *d, uint8_t handle[64]);
+void dist_p2p_attach(Dist *d, int side, const uint8_t handle[64]);
+void dist_p2p_attach_local(Dist *d, int side, Dist *peer);
+void dist_p2p_apply_iterated(Dist *d, int T, const double *s, int ns, cudaStream_t stream);
 
 void nccl_unique_id(uint8_t id[128]);
 void *nccl_comm_create(const uint8_t id[128], int nranks, int rank, int device);

@@ -51,7 +51,8 @@ struct Fuse2Geo {
 // FORM 1: Listing 1's 7-point Jacobi (scalars h2inv, a, b), the paper's
 //   7pt-smoother of Table I / Table II, in box27's retimed FORM 1:
 //   T_k = s1_k - 6 s0_k + s0_{k-1}, B[k] = a A[k] - (b h2inv)(T_k + s0_{k+1}).
-template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2, bool ODD = false, int FORM = 0>
+template <int GX, int GY, int UY, int PF, int MINB = 1, int UX = 2, bool ODD = false, int FORM = 0,
+          bool MIR = false>
 __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MINB)
     sdag_box27x2(const __grid_constant__ SweepArgs a) {
     using G = Fuse2Geo<GX, GY, UY, PF, UX, ODD>;
@@ -205,6 +206,7 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
         fold(s1, cc, uu, s0);
         const int k = j - 1;
         double *o = a.out[0] + ((zbase + k) * a.ny + (ry0 + cy)) * a.nx + gi;
+        const bool mp = MIR && mirror_plane(a, k);
 #pragma unroll
         for (int py = 0; py < UY; py++) {
             double res[UX];
@@ -226,9 +228,12 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
                 for (int px = 0; px < UX; px += 2) {
                     if (vec_ok && outm[px] && outm[px + 1]) {
                         __stcs(reinterpret_cast<double2 *>(o + px), make_double2(res[px], res[px + 1]));
+                        if constexpr (MIR) if (mp) mirror2(a, k, o + px, res[px], res[px + 1]);
                     } else {
                         if (outm[px]) __stcs(o + px, res[px]);
                         if (outm[px + 1]) __stcs(o + px + 1, res[px + 1]);
+                        if (MIR && mp && outm[px]) mirror1(a, k, o + px, res[px]);
+                        if (MIR && mp && outm[px + 1]) mirror1(a, k, o + px + 1, res[px + 1]);
                     }
                 }
             }

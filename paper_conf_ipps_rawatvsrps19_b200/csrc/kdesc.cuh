@@ -88,6 +88,7 @@ KernelDesc make_box27_desc(const char *dag, int prio) {
                   PF);
     d.variant = buf;
     d.fn = reinterpret_cast<const void *>(&dev::sdag_box27<TX, TY, UY, PF, TMA, FORM>);
+    d.fn_mirror = reinterpret_cast<const void *>(&dev::sdag_box27<TX, TY, UY, PF, TMA, FORM, true>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = TX;
@@ -285,6 +286,7 @@ KernelDesc make_fuse2_desc(const char *dag, int prio) {
         std::snprintf(buf, sizeof buf, "%s_tma_%dx%d_u%dx%d_pf%d", tag, GX - 2, GY - 2, UX, UY, PF);
     d.variant = buf;
     d.fn = reinterpret_cast<const void *>(&dev::sdag_box27x2<GX, GY, UY, PF, MINB, UX, ODD, FORM>);
+    d.fn_mirror = reinterpret_cast<const void *>(&dev::sdag_box27x2<GX, GY, UY, PF, MINB, UX, ODD, FORM, true>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = GX - 2;
@@ -316,6 +318,7 @@ KernelDesc make_fuseN_desc(const char *dag, int prio) {
                   UX, UY, PF, MINB);
     d.variant = buf;
     d.fn = reinterpret_cast<const void *>(&dev::sdag_boxfuse<NT, GX, GY, UY, PF, MINB, UX, ODD, FORM>);
+    d.fn_mirror = reinterpret_cast<const void *>(&dev::sdag_boxfuse<NT, GX, GY, UY, PF, MINB, UX, ODD, FORM, true>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = GX - 2 * H;

@@ -19,6 +19,7 @@ struct KernelDesc {
     int nin = 0, nout = 0, nio = 0, n1d = 0;
     int rz = 0, ry = 0, rx = 0, rzr = 0;  // body radius and shared-memory ring z-window
     int prio = 0;                         // heuristic preference (lower first)
+    const void *fn_mirror = nullptr;      // same kernel, also storing into SweepArgs::peer (dist p2p halo)
     int tsteps = 1;                       // sweeps fused per launch (temporal fusion, NEXT-1)
     double fhint = 0.0;                   // measured f(x): launch cost / one sweep (0 = generic estimate)
     std::vector<std::pair<int, int>> inbox;  // per staged input: TMA box (x, y) if cropped (else tx+2rx, ty+2ry)

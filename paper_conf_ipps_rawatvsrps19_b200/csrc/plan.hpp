@@ -92,11 +92,27 @@ void program_apply(Program *g, double *const *a3, int n3, const double *const *a
                    int batch, cudaStream_t stream);
 void plan_fill_info(Plan *p, sdag_plan_info *info);
 
+// Peer-memory halo of one launch (dist p2p path): output planes [klo[s], khi[s])
+// are also stored into neighbour s's buffer `peer[s]` at element offset
+// `off[s]` (same layout); launches KernelDesc::fn_mirror.
+struct Mirror {
+    double *peer[2] = {nullptr, nullptr};
+    int64_t off[2] = {0, 0};
+    int32_t klo[2] = {0, 0}, khi[2] = {0, 0};
+};
+
 // sweep launch over output planes [klo, khi) of each problem (clipped to the
 // interior); all arrays are per-problem [batch][nz][ny][nx].
 void plan_launch(Plan *p, const KernelDesc &k, double *const *arrays3d, const double *const *arrays1d,
                  const double *scalars, int batch, int64_t klo, int64_t khi, cudaStream_t stream,
-                 const int64_t *dims_override = nullptr, const int64_t *zr = nullptr);
+                 const int64_t *dims_override = nullptr, const int64_t *zr = nullptr, const Mirror *mir = nullptr);
+
+// dist p2p synchronisation (p2p.cu): wait until flags[s] - need[s] >= 0 (mod 2^32)
+// for the sides with has[s]; then signal: store v into f0 / f1 (non-null) with
+// system-scope release after the stream's previous work.
+void p2p_wait(const uint32_t *flags, const uint32_t need[2], const int has[2], cudaStream_t stream);
+void p2p_signal(uint32_t *f0, uint32_t *f1, uint32_t v, cudaStream_t stream);
+void p2p_preload();
 void apply(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns, int batch,
            cudaStream_t stream);
 // the argument checks of apply (counts, nulls, output aliasing), nothing enqueued

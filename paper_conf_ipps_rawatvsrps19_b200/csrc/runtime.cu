@@ -208,7 +208,8 @@ static const KernelDesc &pick_kernel(Plan *p, double *const *a3, int64_t nx) {
 }
 
 void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *const *a1, const double *s, int batch,
-                 int64_t klo, int64_t khi, cudaStream_t stream, const int64_t *dims_override, const int64_t *zr) {
+                 int64_t klo, int64_t khi, cudaStream_t stream, const int64_t *dims_override, const int64_t *zr,
+                 const Mirror *mir) {
     const int64_t *dims = dims_override ? dims_override : p->dims;
     int64_t lo[3], hi[3];
     for (int a = 0; a < 3; a++) {
@@ -253,6 +254,17 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *
     // local position
     A.zr_lo = int32_t(zr ? zr[0] : lo[0]);
     A.zr_hi = int32_t(zr ? zr[1] : hi[0]);
+    const bool use_mirror = mir && (mir->peer[0] || mir->peer[1]);
+    if (use_mirror) {
+        if (!k.fn_mirror || k.fission || batch != 1)
+            throw Error(SDAG_ERR_UNSUPPORTED, "kernel " + k.variant + " cannot store into peer memory");
+        for (int q = 0; q < 2; q++) {
+            A.peer[q] = mir->peer[q];
+            A.peer_off[q] = mir->off[q];
+            A.peer_klo[q] = mir->klo[q];
+            A.peer_khi[q] = mir->khi[q];
+        }
+    }
     A.lo[0] = int32_t(klo);
     A.hi[0] = int32_t(khi);
     for (int a = 1; a < 3; a++) {
@@ -279,7 +291,7 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *
     // each evaluating only that output (shared temporaries replicated)
     const int nlaunch = k.fission ? int(k.fission_fns.size()) : 1;
     for (int q = 0; q < nlaunch; q++) {
-        const void *fn = k.fission ? k.fission_fns[q] : k.fn;
+        const void *fn = k.fission ? k.fission_fns[q] : (use_mirror ? k.fn_mirror : k.fn);
         if (!k.cufn) {
             std::lock_guard<std::mutex> g(attr_mu);
             int &d = attr_done[fn];

@@ -67,7 +67,34 @@ struct SweepArgs {
     int32_t tiles_x, tiles_y, nchunk, zchunk;
     int32_t xmin;                 // first interior x (lo[2] may be rounded down to even as tile origin)
     int32_t zr_lo, zr_hi;         // multi-sweep kernels: planes [zr_lo, zr_hi) are global interior (others ring)
+    // peer-memory halo (dist p2p path): output plane k in [peer_klo[s], peer_khi[s])
+    // is also stored into z-neighbour s's buffer at element offset
+    // (o - out[0]) + peer_off[s] (s = 0 lower, 1 upper; null = none)
+    double *peer[2];
+    int64_t peer_off[2];
+    int32_t peer_klo[2], peer_khi[2];
 };
+
+// Store-side fusion of the z-slab halo exchange: a
+// kernel that writes output plane k also writes it, over NVLink P2P, into the
+// ghost band of the neighbour that reads it next sweep.
+// true iff output plane k goes to a neighbour too (uniform per plane: test it
+// once, outside the store loop, so the common path carries no per-store checks)
+__device__ __forceinline__ bool mirror_plane(const SweepArgs &a, int k) {
+    return (a.peer[0] && k >= a.peer_klo[0] && k < a.peer_khi[0]) ||
+           (a.peer[1] && k >= a.peer_klo[1] && k < a.peer_khi[1]);
+}
+__device__ __forceinline__ void mirror2(const SweepArgs &a, int k, const double *o, double x, double y) {
+#pragma unroll
+    for (int s = 0; s < 2; s++)
+        if (a.peer[s] && k >= a.peer_klo[s] && k < a.peer_khi[s])
+            __stcs(reinterpret_cast<double2 *>(a.peer[s] + (o - a.out[0]) + a.peer_off[s]), make_double2(x, y));
+}
+__device__ __forceinline__ void mirror1(const SweepArgs &a, int k, const double *o, double v) {
+#pragma unroll
+    for (int s = 0; s < 2; s++)
+        if (a.peer[s] && k >= a.peer_klo[s] && k < a.peer_khi[s]) __stcs(a.peer[s] + (o - a.out[0]) + a.peer_off[s], v);
+}
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
