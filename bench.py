@@ -257,6 +257,118 @@ def run_other(args):
     return 0
 
 
+def run_slabs27(args):
+    """Config 5 as BASELINE names it: the iterated 27-point smoother, 1024^3 per
+    GPU, T = 12 sweeps per step, weak-scaled as z-slabs (one rank per GPU).
+    --halo nccl: ghost planes exchanged by NCCL send/recv on a comm stream,
+    overlapped with the interior launch (sdag_dist_apply_iterated);
+    --halo p2p: the boundary launches store their planes straight into the
+    neighbours' ghost planes over NVLink (sdag_dist_p2p_apply_iterated; CUDA IPC
+    handles exchanged over the process group), no NCCL.  Ghost depth 2 R_z
+    (time_tile 2): one exchange per fused 2-sweep launch.
+    SDAG_BENCH_SAME_DEVICE=1 maps every rank to cuda:0 (plumbing check of the
+    multi-process p2p path on one GPU; times are then not scaling numbers)."""
+    import torch
+    import torch.distributed as tdist
+    import paper_conf_ipps_rawatvsrps19_b200 as sdag
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = 0 if os.environ.get("SDAG_BENCH_SAME_DEVICE") else int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    halo = args.halo or "nccl"
+    pg = None
+    if world > 1:
+        if halo == "p2p":
+            tdist.init_process_group("gloo")  # host plumbing only: IPC handles, barrier, timing reduce
+        else:
+            tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        pg = tdist
+    name, T, tt = "smooth27", 12, 2
+    spec = sdag.spec_text(name)
+    n = int(os.environ.get("SDAG_BENCH_SLAB_N", "1024"))
+    gdims = (n * world, n, n)
+    scal = [-128 / 30, 14 / 30, 3 / 30, 1 / 30, 0.125]
+    comm = None
+    if halo == "nccl" and world > 1:
+        uid = [sdag.nccl_unique_id() if rank == 0 else None]
+        tdist.broadcast_object_list(uid, src=0)
+        comm = sdag.nccl_comm_create(uid[0], world, rank, local)
+    dd = sdag.Dist(spec, gdims, rank, world, comm=comm, time_tile=tt, variant=args.variant)
+    (nza, ny, nx), g0 = dd.layout()
+    part = sdag.slab_partition2(gdims[0], 1, tt, world, rank)
+    stream = torch.cuda.current_stream()
+    full = torch.from_numpy(__import__("synth").uniform((nza, ny, nx), -1.0, 1.0, "cfg5-slab", rank))
+    if halo == "p2p":
+        b0, b1 = dd.p2p_alloc()
+        b0.copy_(full)
+        b1.copy_(full)
+        torch.cuda.synchronize()
+        if world > 1:
+            hs = [None] * world
+            tdist.all_gather_object(hs, dd.p2p_handle())
+            if rank > 0:
+                dd.p2p_attach(0, hs[rank - 1])
+            if rank < world - 1:
+                dd.p2p_attach(1, hs[rank + 1])
+
+        def step():
+            dd.p2p_apply_iterated(T, scalars=scal, stream=stream)
+    else:
+        b0 = full.cuda()
+        b1 = b0.clone()
+        cs = torch.cuda.Stream()
+
+        def step():
+            dd.apply_iterated(b0, b1, T, scalars=scal, stream=stream, comm_stream=cs)
+    del full
+    info = dd.plan.info
+    pts_rank = (part["k_hi"] - part["k_lo"]) * (ny - 2) * (nx - 2) * T
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if pg:
+        tdist.barrier()
+    l0 = sdag.launch_count()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with Clocks(local) as clk:
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(args.steps):
+            step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+    launches = sdag.launch_count() - l0
+    ms = e0.elapsed_time(e1)
+    red = torch.tensor([ms, float(pts_rank)], dtype=torch.float64)
+    if pg:
+        tdist.barrier()
+        mx = red.clone()
+        tdist.all_reduce(mx, op=tdist.ReduceOp.MAX)
+        sm = red.clone()
+        tdist.all_reduce(sm, op=tdist.ReduceOp.SUM)
+        ms_max, total_pts = float(mx[0]), float(sm[1])
+    else:
+        ms_max, total_pts = ms, float(pts_rank)
+    flops = total_pts * info["flops_per_point"] * args.steps
+    if rank == 0:
+        line = {"metric": METRIC, "value": flops / (ms_max * 1e-3) / 1e9, "unit": "GFLOP/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic (counter-based generator, per-rank slab)",
+                "config": {"workload": CONFIGS[name][2], "stencil": name, "grid_per_gpu": [n, n, n],
+                           "global_grid": list(gdims), "decomposition": f"z-slabs x{world}", "halo": halo,
+                           "time_tile": tt, "sweeps_per_step": T, "variant": info["variant"],
+                           "same_device": bool(os.environ.get("SDAG_BENCH_SAME_DEVICE")),
+                           "l2": "8 GiB slab/GPU > 126 MB L2 (no flush needed)"},
+                "hbm_gbs_sweep_equivalent": total_pts * info["bytes_per_point"] * args.steps / (ms_max * 1e-3) / 1e9,
+                "gpu_launches": launches, "clocks": clk.summary()}
+        print(json.dumps(line))
+    if pg:
+        tdist.barrier()
+        tdist.destroy_process_group()
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -271,10 +383,15 @@ def main():
                     help="take the z-slab/NCCL path even on one rank (plumbing check of the multi-GPU code)")
     ap.add_argument("--config", default="lap25", choices=list(CONFIGS),
                     help="lap25 = the headline line; the others record the remaining BASELINE stencils (N=1)")
+    ap.add_argument("--halo", default=None, choices=["nccl", "p2p"],
+                    help="with --config smooth27: the z-slab run of config 5 (BASELINE's multi-GPU workload) "
+                         "with this halo path")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
         return run_reference(args)
+    if args.config == "smooth27" and (args.halo or int(os.environ.get("WORLD_SIZE", "1")) > 1):
+        return run_slabs27(args)
     if args.config != "lap25":
         return run_other(args)
 
