@@ -337,6 +337,30 @@ sdag_status sdag_dist_p2p_apply_iterated(sdag_dist d, int32_t T, const double *s
                                          sdag_stream stream);
 
 /* ------------------------------------------------------------------------
+ * Profile-guided classification (paper Section IV)
+ * ------------------------------------------------------------------------ */
+enum { SDAG_BOUND_DRAM = 0, SDAG_BOUND_COMPUTE = 1, SDAG_BOUND_LATENCY = 2 };
+typedef struct {
+    char variant[96];          /* the plan's kernel */
+    double ms;                 /* median of 7 timed launches on the caller's arrays */
+    double flops, bytes;       /* canonical flops, algorithmic bytes of one apply (R9, R10) */
+    double oi_dram, ridge;     /* flops/bytes; peak_fp64 / peak_hbm (flop/B) */
+    double peak_hbm_gbs, peak_fp64_tflops;  /* as passed, or measured (copy, DFMA) when 0 */
+    double frac_dram, frac_fp64;            /* roofline time of each level / ms */
+    double ms_diff_mem, ms_diff_arith;      /* code-differenced twins, 0 if none */
+    int32_t regs, spill_bytes, ctas_per_sm, warps_per_sm;
+    int32_t bound;             /* SDAG_BOUND_* */
+    char hints[1024];          /* Section IV-A guidelines applied to this plan, '\n'-separated */
+} sdag_profile;
+/* Runs the plan's kernel on the caller's arrays (same arguments as sdag_apply;
+ * the outputs are overwritten several times) and classifies it.  Synchronous
+ * on `stream`.  peak_* <= 0: measured here (a 1 GiB device copy, the DFMA
+ * micro-benchmark).  Errors as sdag_apply. */
+sdag_status sdag_plan_profile(sdag_plan plan, void *const *arrays3d, int32_t n3d, const double *const *arrays1d,
+                              int32_t n1d, const double *scalars, int32_t nscalars, double peak_hbm_gbs,
+                              double peak_fp64_tflops, sdag_stream stream, sdag_profile *out);
+
+/* ------------------------------------------------------------------------
  * Diagnostics
  * ------------------------------------------------------------------------ */
 const char *sdag_last_error(void); /* thread-local; valid until the next sdag_* call on this thread */

@@ -181,6 +181,23 @@ class Plan:
         return self._L.sdag_plan_describe(self._h).decode()
 
     # ---- apply ----
+    def profile(self, arrays3d, arrays1d=(), scalars=(), peak_hbm_gbs=0.0, peak_fp64_tflops=0.0, stream=None):
+        """Profile-guided classification (paper Section IV): the plan's kernel timed on
+        these arrays, its DRAM / FP64 roofline fractions, code-differenced twins,
+        resources, the bound (dram | compute | latency) and the Section IV-A hints.
+        Overwrites the outputs; synchronous."""
+        p3 = [_ptr(t, "grid array") for t in arrays3d]
+        p1 = [_ptr(t, "1D array") for t in arrays1d]
+        s, ns = _scal(scalars)
+        pr = _capi.Profile()
+        _check(self._L.sdag_plan_profile(self._h, _arr(p3), len(p3), _arr(p1), len(p1), s, ns, float(peak_hbm_gbs),
+                                         float(peak_fp64_tflops), _stream_handle(stream), ctypes.byref(pr)))
+        d = {k: getattr(pr, k) for k, _ in _capi.Profile._fields_}
+        d["variant"] = pr.variant.decode()
+        d["hints"] = [h for h in pr.hints.decode().split("\n") if h]
+        d["bound"] = {0: "dram", 1: "compute", 2: "latency"}[pr.bound]
+        return d
+
     def apply(self, arrays3d, arrays1d=(), scalars=(), stream=None):
         p3 = [_ptr(t, "grid array") for t in arrays3d]
         p1 = [_ptr(t, "1D array") for t in arrays1d]

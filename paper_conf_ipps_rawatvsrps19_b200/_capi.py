@@ -89,6 +89,8 @@ def lib():
             "sdag_dist_apply_iterated_loopback": (S, [ctypes.POINTER(P), c_i32, ctypes.POINTER(c_void_p),
                                                       ctypes.POINTER(c_void_p), c_i32, c_dblp, c_i32, P]),
             "sdag_dist_destroy": (None, [P]),
+            "sdag_plan_profile": (S, [P, ctypes.POINTER(c_void_p), c_i32, ctypes.POINTER(c_void_p), c_i32, c_dblp,
+                                      c_i32, ctypes.c_double, ctypes.c_double, P, ctypes.c_void_p]),
             "sdag_dist_p2p_alloc": (S, [P, ctypes.POINTER(c_void_p), ctypes.POINTER(c_void_p)]),
             "sdag_dist_p2p_handle": (S, [P, ctypes.c_char_p]),
             "sdag_dist_p2p_attach": (S, [P, c_i32, ctypes.c_char_p]),
@@ -109,6 +111,17 @@ def lib():
     return _lib
 
 
+class Profile(ctypes.Structure):
+    """sdag_profile (include/sdag.h)"""
+    _fields_ = [("variant", ctypes.c_char * 96), ("ms", ctypes.c_double), ("flops", ctypes.c_double),
+                ("bytes", ctypes.c_double), ("oi_dram", ctypes.c_double), ("ridge", ctypes.c_double),
+                ("peak_hbm_gbs", ctypes.c_double), ("peak_fp64_tflops", ctypes.c_double),
+                ("frac_dram", ctypes.c_double), ("frac_fp64", ctypes.c_double),
+                ("ms_diff_mem", ctypes.c_double), ("ms_diff_arith", ctypes.c_double),
+                ("regs", ctypes.c_int32), ("spill_bytes", ctypes.c_int32), ("ctas_per_sm", ctypes.c_int32),
+                ("warps_per_sm", ctypes.c_int32), ("bound", ctypes.c_int32), ("hints", ctypes.c_char * 1024)]
+
+
 # every symbol include/sdag.h declares (checked by tests/test_capi_symbols.py)
 EXPORTED = [
     "sdag_plan_opts_init", "sdag_plan_create", "sdag_plan_info_get", "sdag_plan_arg", "sdag_plan_variant_name",
@@ -119,7 +132,7 @@ EXPORTED = [
     "sdag_slab_partition2", "sdag_slab_halo2", "sdag_nccl_get_unique_id", "sdag_nccl_comm_create",
     "sdag_nccl_comm_destroy", "sdag_dist_create", "sdag_dist_layout", "sdag_dist_local_plan", "sdag_dist_apply",
     "sdag_dist_apply_iterated", "sdag_dist_destroy", "sdag_dist_apply_iterated_loopback",
-    "sdag_dist_p2p_alloc", "sdag_dist_p2p_handle", "sdag_dist_p2p_attach", "sdag_dist_p2p_attach_local",
+    "sdag_plan_profile", "sdag_dist_p2p_alloc", "sdag_dist_p2p_handle", "sdag_dist_p2p_attach", "sdag_dist_p2p_attach_local",
     "sdag_dist_p2p_apply_iterated", "sdag_last_error",
     "sdag_version", "sdag_launch_count", "sdag_measure_fp64_peak", "sdag_registry_count", "sdag_registry_get",
 ]

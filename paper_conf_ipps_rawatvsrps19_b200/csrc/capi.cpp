@@ -328,6 +328,16 @@ sdag_status sdag_dist_apply_iterated_loopback(sdag_dist *dists, int32_t nranks, 
 
 void sdag_dist_destroy(sdag_dist d) { delete reinterpret_cast<sdag::Dist *>(d); }
 
+sdag_status sdag_plan_profile(sdag_plan plan, void *const *a3, int32_t n3, const double *const *a1, int32_t n1,
+                              const double *s, int32_t ns, double peak_hbm_gbs, double peak_fp64_tflops,
+                              sdag_stream stream, sdag_profile *out) {
+    return guard([&] {
+        if (!plan || !plan->p) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null plan");
+        sdag::plan_profile(plan->p, reinterpret_cast<double *const *>(a3), n3, a1, n1, s, ns, peak_hbm_gbs,
+                           peak_fp64_tflops, reinterpret_cast<cudaStream_t>(stream), out);
+    });
+}
+
 sdag_status sdag_dist_p2p_alloc(sdag_dist d, double **buf0, double **buf1) {
     return guard([&] { sdag::dist_p2p_alloc(reinterpret_cast<sdag::Dist *>(d), buf0, buf1); });
 }

@@ -113,6 +113,8 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *arrays3d, const do
 void p2p_wait(const uint32_t *flags, const uint32_t need[2], const int has[2], cudaStream_t stream);
 void p2p_signal(uint32_t *f0, uint32_t *f1, uint32_t v, cudaStream_t stream);
 void p2p_preload();
+void plan_profile(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns,
+                  double peak_hbm_gbs, double peak_fp64_tflops, cudaStream_t st, sdag_profile *out);
 void apply(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns, int batch,
            cudaStream_t stream);
 // the argument checks of apply (counts, nulls, output aliasing), nothing enqueued

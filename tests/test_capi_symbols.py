@@ -40,3 +40,12 @@ def test_library_is_sm100a_only():
 def test_version_and_launch_counter():
     assert "sm_100a" in sdag.version()
     assert sdag.launch_count() >= 0
+
+
+def test_profile_struct_layout():
+    """ctypes mirror of sdag_profile: 96-byte name, 11 doubles, 5 int32, 1024-byte hints"""
+    import ctypes
+
+    from paper_conf_ipps_rawatvsrps19_b200 import _capi
+    assert _capi.Profile.hints.offset == 96 + 11 * 8 + 5 * 4
+    assert ctypes.sizeof(_capi.Profile) == 96 + 11 * 8 + 5 * 4 + 1024 + 4  # padded to 8
