@@ -11,7 +11,7 @@ ARCH    := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -Wall -Iinclude -I$(SRC) -I$(BUILD) \
            --expt-relaxed-constexpr
 CU_SRCS := k_jacobi7 k_lap25 k_smooth27 k_hypterm k_rhs4 k_toys runtime jit p2p profile
-CC_SRCS := spec analysis registry dist capi program
+CC_SRCS := spec analysis registry dist capi program fission
 OBJS    := $(addprefix $(BUILD)/,$(addsuffix .o,$(CU_SRCS) $(CC_SRCS)))
 HDRS    := $(wildcard $(SRC)/*.hpp $(SRC)/*.cuh) include/sdag.h
 

@@ -337,6 +337,25 @@ sdag_status sdag_dist_p2p_apply_iterated(sdag_dist d, int32_t T, const double *s
                                          sdag_stream stream);
 
 /* ------------------------------------------------------------------------
+ * Fission (paper Section VI-B): split versions written out as DSL
+ * ------------------------------------------------------------------------ */
+enum { SDAG_FISSION_MAXFUSE = 0, SDAG_FISSION_TRIVIAL = 1 };
+/* From a single-stage spec, the DSL text of a split version, accepted by
+ * sdag_program_create with the same arguments (declaration order = the
+ * stencil's formal order):
+ *   SDAG_FISSION_MAXFUSE: the stencil re-printed from the IR (one stage);
+ *   SDAG_FISSION_TRIVIAL: one stencil function per output array with the
+ *     statements it needs (temporaries replicated, Fig 3b/3c), called in an
+ *     order that preserves every value a statement reads; UNSUPPORTED if no
+ *     such order exists.
+ * Statements are selected, not rewritten (parenthesised trees, exact
+ * literals), so each output is computed by the same operations.  *len = text
+ * length (without the NUL); the text is copied into buf when cap > *len, and
+ * INVALID_ARG is returned when buf is non-null and too small.  Parse and
+ * semantic errors as sdag_plan_create.  Host only. */
+sdag_status sdag_spec_fission(const char *spec, int32_t kind, char *buf, int64_t cap, int64_t *len);
+
+/* ------------------------------------------------------------------------
  * Profile-guided classification (paper Section IV)
  * ------------------------------------------------------------------------ */
 enum { SDAG_BOUND_DRAM = 0, SDAG_BOUND_COMPUTE = 1, SDAG_BOUND_LATENCY = 2 };

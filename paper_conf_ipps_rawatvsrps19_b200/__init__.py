@@ -21,7 +21,7 @@ import os
 from . import _capi
 from ._capi import PlanInfo, PlanOpts, SDAG_DEVICE_CURRENT, SDAG_DEVICE_NONE
 
-__all__ = ["Plan", "Program", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "slab_partition2", "slab_halo2", "nccl_unique_id",
+__all__ = ["Plan", "Program", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "slab_partition2", "slab_halo2", "fission", "nccl_unique_id",
            "nccl_comm_create", "nccl_comm_destroy", "launch_count", "fp64_peak", "version", "SPEC_DIR"]
 
 SPEC_DIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "specs")
@@ -451,6 +451,19 @@ class _DeviceView:
     def __init__(self, ptr, shape):
         self.__cuda_array_interface__ = {"shape": shape, "typestr": "<f8", "data": (int(ptr), False),
                                          "version": 3, "strides": None}
+
+
+def fission(spec: str, kind: str = "trivial") -> str:
+    """The paper's fission versions (Section VI-B) of a single-stage spec as DSL
+    text for Program: kind "trivial" (one stencil per output, Fig 3c) or
+    "maxfuse" (the stencil re-printed)"""
+    k = {"maxfuse": 0, "trivial": 1}[kind]
+    L = _capi.lib()
+    n = ctypes.c_int64()
+    _check(L.sdag_spec_fission(spec.encode(), k, None, 0, ctypes.byref(n)))
+    buf = ctypes.create_string_buffer(n.value + 1)
+    _check(L.sdag_spec_fission(spec.encode(), k, buf, n.value + 1, ctypes.byref(n)))
+    return buf.value.decode()
 
 
 def launch_count() -> int:

@@ -1,0 +1,251 @@
+// fission.cpp -- the paper's fission component (Section VI-B):
+// from a single-stage spec, write the split versions back out as DSL text that
+// sdag_program_create accepts (ARTEMIS "writes them out as DSL specification
+// files"):
+//   * maxfuse: the stencil itself, re-printed from the IR (every stencil
+//     function with the same domain fused -- one stage here);
+//   * trivial-fission: one stencil function per output array, holding the
+//     statements that array needs (temporaries replicated, Fig 3b/3c), called
+//     in an order that preserves every value a statement reads.
+// A split is emitted only if every stage keeps the stencil's radius (each
+// stage's output domain is the interior of its own radius, reading R1).
+// Recompute-fission splits outputs so that each kernel's recomputation halo is
+// <= max(4, r); the temporaries of this DSL are per-point scalars (reading
+// R15), so a single stage has no recomputation halo and recompute-fission
+// coincides with maxfuse.
+//
+// Statements are selected, never rewritten: each printed expression is the
+// parsed tree, fully parenthesised, literals printed to round-trip exactly.
+#include <algorithm>
+#include <cstdio>
+#include <set>
+#include <sstream>
+
+#include "ir.hpp"
+#include "sdag.h"
+
+namespace sdag {
+
+namespace {
+
+std::string num(double v) {
+    char b[40];
+    std::snprintf(b, sizeof b, "%.17g", v);
+    std::string s = b;
+    if (s.find_first_of(".eEn") == std::string::npos) s += ".0";  // a double literal
+    return s;
+}
+
+struct Printer {
+    const Stencil &st;
+    std::string expr(int n) const {
+        const Node &x = st.nodes[n];
+        switch (x.kind) {
+            case Node::Num: return num(x.value);
+            case Node::Scalar: return st.formal(ArgKind::Scalar, x.ref).name;
+            case Node::Temp: return st.temps[x.ref];
+            case Node::Load3: {
+                std::string s = st.formal(ArgKind::Array3D, x.ref).name;
+                for (int a = 0; a < 3; a++) s += "[" + idx(a, x.off[a]) + "]";
+                return s;
+            }
+            case Node::Load1: {
+                const Formal &f = st.formal(ArgKind::Array1D, x.ref);
+                return f.name + "[" + idx(f.axis, x.off[0]) + "]";
+            }
+            case Node::Neg: return "(-" + expr(x.a) + ")";
+            case Node::Add: return "(" + expr(x.a) + " + " + expr(x.b) + ")";
+            case Node::Sub: return "(" + expr(x.a) + " - " + expr(x.b) + ")";
+            case Node::Mul: return "(" + expr(x.a) + " * " + expr(x.b) + ")";
+            case Node::Div: return "(" + expr(x.a) + " / " + expr(x.b) + ")";
+        }
+        throw Error(SDAG_ERR_INVALID_ARG, "fission: unknown node");
+    }
+    std::string idx(int axis, int off) const {
+        const std::string &it = st.iterators[axis];
+        if (off == 0) return it;
+        return it + (off > 0 ? "+" : "-") + std::to_string(std::abs(off));
+    }
+};
+
+// temporaries and 3D arrays (offset 0 reads) an expression reads
+void reads(const Stencil &st, int n, std::set<int> &temps, std::vector<int> *arrays0) {
+    const Node &x = st.nodes[n];
+    if (x.kind == Node::Temp) temps.insert(x.ref);
+    if (x.kind == Node::Load3 && arrays0 && x.off[0] == 0 && x.off[1] == 0 && x.off[2] == 0)
+        arrays0->push_back(x.ref);
+    if (x.a >= 0) reads(st, x.a, temps, arrays0);
+    if (x.b >= 0) reads(st, x.b, temps, arrays0);
+}
+
+// per-axis radius of the reads of an expression (3D and 1D, reading R2)
+void radius_of(const Stencil &st, int n, int r[3]) {
+    const Node &x = st.nodes[n];
+    if (x.kind == Node::Load3)
+        for (int a = 0; a < 3; a++) r[a] = std::max(r[a], std::abs(x.off[a]));
+    if (x.kind == Node::Load1) {
+        const int a = st.formal(ArgKind::Array1D, x.ref).axis;
+        if (a >= 0) r[a] = std::max(r[a], std::abs(x.off[0]));
+    }
+    if (x.a >= 0) radius_of(st, x.a, r);
+    if (x.b >= 0) radius_of(st, x.b, r);
+}
+
+std::string header(const Stencil &st) {
+    std::ostringstream o;
+    o << "iterator";
+    for (size_t a = 0; a < st.iterators.size(); a++) o << (a ? ", " : " ") << st.iterators[a];
+    o << ";\n";
+    // declared extents are placeholders: a plan's extents come from sdag_plan_create
+    std::vector<std::string> decl;
+    std::set<std::string> seen;
+    for (const Formal &f : st.formals) {
+        const std::string &n = f.actual.empty() ? f.name : f.actual;
+        if (!seen.insert(n).second) continue;
+        if (f.kind == ArgKind::Array3D)
+            decl.push_back(n + "[64,64,64]");
+        else if (f.kind == ArgKind::Array1D)
+            decl.push_back(n + "[64]");
+        else
+            decl.push_back(n);
+    }
+    o << "double";
+    for (size_t q = 0; q < decl.size(); q++) o << (q ? ", " : " ") << decl[q];
+    o << ";\n";
+    return o.str();
+}
+
+std::string formals_list(const Stencil &st, bool actual) {
+    std::string s = "(";
+    for (size_t q = 0; q < st.formals.size(); q++) {
+        const Formal &f = st.formals[q];
+        s += (q ? ", " : "") + ((actual && !f.actual.empty()) ? f.actual : f.name);
+    }
+    return s + ")";
+}
+
+std::string function(const Stencil &st, const std::string &name, const std::vector<bool> &keep) {
+    Printer P{st};
+    std::ostringstream o;
+    o << "stencil " << name << " " << formals_list(st, false) << " {\n";
+    std::set<int> declared;
+    for (size_t q = 0; q < st.stmts.size(); q++) {
+        if (!keep[q]) continue;
+        const Statement &s = st.stmts[q];
+        o << "    ";
+        if (s.to_array) {
+            o << st.formal(ArgKind::Array3D, s.target).name << "[" << P.idx(0, 0) << "][" << P.idx(1, 0) << "]["
+              << P.idx(2, 0) << "]";
+        } else {
+            if (declared.insert(s.target).second) o << "double ";
+            o << st.temps[s.target];
+        }
+        o << " = " << P.expr(s.expr) << ";\n";
+    }
+    o << "}\n";
+    return o.str();
+}
+
+}  // namespace
+
+std::string emit_fission(const std::string &spec, int kind) {
+    const Stencil st = parse_spec(spec);
+    (void)analyse(st);  // the spec must be a valid single-stage DAG
+    const int ns = int(st.stmts.size());
+    if (kind == 0) {  // maxfuse: the stencil re-printed
+        std::vector<bool> all(ns, true);
+        return header(st) + function(st, st.name, all) + st.name + " " + formals_list(st, true) + ";\n";
+    }
+    if (kind != 1) throw Error(SDAG_ERR_INVALID_ARG, "fission kind must be 0 (maxfuse) or 1 (trivial-fission)");
+
+    // output arrays in order of first write
+    std::vector<int> outs;
+    for (const Statement &s : st.stmts)
+        if (s.to_array && std::find(outs.begin(), outs.end(), s.target) == outs.end()) outs.push_back(s.target);
+    const int no = int(outs.size());
+    auto out_index = [&](int arr) {
+        auto it = std::find(outs.begin(), outs.end(), arr);
+        return it == outs.end() ? -1 : int(it - outs.begin());
+    };
+
+    // backward slice per output: keep its writes and, by liveness, the
+    // temporary assignments whose values they (transitively) read
+    std::vector<std::vector<bool>> keep(no, std::vector<bool>(ns, false));
+    std::vector<std::set<int>> before(no);  // kernels that must run before kernel m
+    for (int m = 0; m < no; m++) {
+        std::set<int> live;
+        for (int q = ns - 1; q >= 0; q--) {
+            const Statement &s = st.stmts[q];
+            const bool writes_out = s.to_array && s.target == outs[m];
+            const bool defines_live = !s.to_array && live.count(s.target);
+            if (!writes_out && !defines_live) continue;
+            keep[m][q] = true;
+            if (defines_live) live.erase(s.target);
+            reads(st, s.expr, live, nullptr);
+        }
+        // value-order constraints: a kept statement reading another output X
+        // at the point sees X's new value if X was written earlier in program
+        // order (X's kernel must run first), else its old value (X's kernel
+        // must run after this one)
+        for (int q = 0; q < ns; q++) {
+            if (!keep[m][q]) continue;
+            std::set<int> tmp;
+            std::vector<int> arrs;
+            reads(st, st.stmts[q].expr, tmp, &arrs);
+            for (int x : arrs) {
+                const int j = out_index(x);
+                if (j < 0 || j == m) continue;
+                bool written_before = false;
+                for (int r = 0; r < q; r++)
+                    if (st.stmts[r].to_array && st.stmts[r].target == x) written_before = true;
+                if (written_before)
+                    before[m].insert(j);
+                else
+                    before[j].insert(m);
+            }
+        }
+    }
+    // each stage's output domain is the interior of ITS radius (reading R1):
+    // a stage that reads less far than the fused stencil would write a wider
+    // domain, so the split is only emitted when every stage keeps the radius
+    const Analysis full = analyse(st);
+    for (int m = 0; m < no; m++) {
+        int r[3] = {0, 0, 0};
+        for (int q = 0; q < ns; q++)
+            if (keep[m][q]) radius_of(st, st.stmts[q].expr, r);
+        for (int a = 0; a < 3; a++)
+            if (r[a] != full.radius[a])
+                throw Error(SDAG_ERR_UNSUPPORTED,
+                            "trivial fission would change the output domain of '" +
+                                st.formal(ArgKind::Array3D, outs[m]).name + "' (its statements read radius " +
+                                std::to_string(r[a]) + " along axis " + std::to_string(a) + ", the stencil " +
+                                std::to_string(full.radius[a]) + ")");
+    }
+    // call order: outputs' first-write order, subject to the constraints
+    std::vector<int> order;
+    std::vector<bool> placed(no, false);
+    for (int step = 0; step < no; step++) {
+        int pick = -1;
+        for (int m = 0; m < no && pick < 0; m++) {
+            if (placed[m]) continue;
+            bool ready = true;
+            for (int j : before[m]) ready = ready && placed[j];
+            if (ready) pick = m;
+        }
+        if (pick < 0)
+            throw Error(SDAG_ERR_UNSUPPORTED,
+                        "trivial fission would change a value some statement reads (outputs read each other's old "
+                        "and new values)");
+        placed[pick] = true;
+        order.push_back(pick);
+    }
+    std::string text = header(st), calls;
+    for (int m : order) {
+        const std::string name = st.name + "_" + st.formal(ArgKind::Array3D, outs[m]).name;
+        text += function(st, name, keep[m]);
+        calls += name + " " + formals_list(st, true) + ";\n";
+    }
+    return text + calls;
+}
+
+}  // namespace sdag

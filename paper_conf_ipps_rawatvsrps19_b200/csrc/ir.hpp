@@ -124,6 +124,9 @@ struct ProgramIR {
 ProgramIR parse_program(const std::string &text);
 // a2: analyse (throws Error for UNSUPPORTED / SEMANTIC findings).
 Analysis analyse(const Stencil &st);
+// fission versions of a single-stage spec as DSL program text (fission.cpp):
+// kind 0 maxfuse, 1 trivial-fission
+std::string emit_fission(const std::string &spec, int kind);
 // canonical, name-free serialisation used to match registered DAGs
 std::string canonical_form(const Stencil &st);
 
