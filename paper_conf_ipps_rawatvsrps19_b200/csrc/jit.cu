@@ -253,7 +253,27 @@ void jit_build_candidates(Plan *p) {
 
     // tile geometries, preference order (the generic skeleton's best shapes on
     // the registered DAGs: tools/perf_sweep.py); smem decides RZR
-    const Geom geoms[] = {{32, 16, 1, 2, 1}, {64, 8, 1, 1, 1}, {16, 16, 1, 1, 1}};
+    std::vector<Geom> geoms = {{32, 16, 1, 2, 1}, {64, 8, 1, 1, 1}, {16, 16, 1, 1, 1}};
+    // the spec's "#pragma ... block (bx,by) unroll j=u": the user's
+    // thread block and unroll factors become the first candidate geometry
+    // (tile = block x unroll per axis)
+    const Pragma &pr = p->st.pragma;
+    if (pr.block[0] > 0 && p->st.iterators.size() == 3) {
+        auto un = [&](int axis) {
+            auto it = pr.unroll.find(p->st.iterators[axis]);
+            return it == pr.unroll.end() ? 1 : it->second;
+        };
+        const int ux = un(2), uy = un(1), bx = pr.block[0], by = pr.block[1] > 0 ? pr.block[1] : 1;
+        const Geom g{bx * ux, by * uy, ux, uy, 1};
+        if (ux >= 1 && uy >= 1 && ux * uy <= 16 && bx * by >= 32 && bx * by <= 1024) {
+            geoms.erase(std::remove_if(geoms.begin(), geoms.end(),
+                                       [&](const Geom &h) {
+                                           return h.tx == g.tx && h.ty == g.ty && h.ux == g.ux && h.uy == g.uy;
+                                       }),
+                        geoms.end());
+            geoms.insert(geoms.begin(), g);
+        }
+    }
     struct Cand {
         Geom g;
         int rzr;

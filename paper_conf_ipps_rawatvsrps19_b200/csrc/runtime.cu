@@ -734,6 +734,19 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
         for (int x = 1; x < 8; x++)
             if (p->fcost[x] > 0.0) d << " f(" << x << ")=" << p->fcost[x];
     }
+    const Pragma &pr = p->st.pragma;
+    if (pr.block[0] > 0 || !pr.unroll.empty() || pr.occupancy > 0 || !p->st.assign.shmem.empty() ||
+        !p->st.assign.gmem.empty()) {
+        d << "\n  user guidance (#pragma / #assign, P:461-471, P:513-533):";
+        if (pr.block[0] > 0) d << " block(" << pr.block[0] << "," << pr.block[1] << ")";
+        for (auto &u : pr.unroll) d << " unroll " << u.first << "=" << u.second;
+        if (pr.occupancy > 0) d << " occupancy " << pr.occupancy;
+        for (auto &a : p->st.assign.gmem) d << " gmem:" << a;
+        for (auto &a : p->st.assign.shmem) d << " shmem:" << a;
+        d << (p->jit_descs.empty() ? "  -- the registered sm_100a kernel keeps its measured geometry and staging "
+                                     "(force a variant, or variant \"jit\" to generate the guided one)"
+                                   : "  -- block x unroll is the first generated geometry");
+    }
     if (!p->jit_descs.empty())
         d << "\n  jit body (NVRTC, sm_100a, into the sweep.cuh skeleton):\n" << jit_body_source(*p, "JitBody", p->an.radius[0]);
     p->describe_text = d.str();
