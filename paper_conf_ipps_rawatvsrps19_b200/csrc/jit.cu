@@ -66,6 +66,9 @@ struct Gen {
         case Node::Temp: return "t" + std::to_string(x.ref);
         case Node::Load3: {
             const int f = x.ref;
+            if (p.in_slot[f] >= p.n_staged)  // #assign gmem: through L1/L2
+                return "g.gm(" + std::to_string(p.in_slot[f]) + ", " + std::to_string(x.off[0]) + ", " +
+                       std::to_string(x.off[1]) + ", " + std::to_string(x.off[2]) + ")";
             if (p.in_slot[f] >= 0)
                 return "g.at(" + std::to_string(p.in_slot[f]) + ", " + std::to_string(x.off[0]) + ", " +
                        std::to_string(x.off[1]) + ", " + std::to_string(x.off[2]) + ")";
@@ -89,7 +92,7 @@ struct Gen {
 
 // The body struct for the sweep skeleton (interface: sweep.cuh header).
 std::string jit_body_source(const Plan &p, const std::string &sname, int rzr) {
-    const int nin = p.an.n_in, nout = p.an.n_out + p.an.n_inout, nio = p.an.n_inout, n1 = p.n1();
+    const int nin = p.n_staged, nout = p.an.n_out + p.an.n_inout, nio = p.an.n_inout, n1 = p.n1();
     std::ostringstream o;
     o << "struct " << sname << " {\n"
       << "    static constexpr int NIN = " << nin << ", NOUT = " << nout << ", NIO = " << nio << ", N1D = " << n1
@@ -243,8 +246,8 @@ struct Geom {
 // plan's DAG.  Throws UNSUPPORTED when the DAG exceeds the skeleton's limits.
 void jit_build_candidates(Plan *p) {
     using namespace dev;
-    const int nin = p->an.n_in, nout = p->an.n_out + p->an.n_inout, nio = p->an.n_inout, n1 = p->n1();
-    if (nin < 1 || nin > MAXIN || nout > MAXOUT || nio > MAXIO || n1 > MAX1D || p->ns() > MAXS)
+    const int nin_all = p->an.n_in, nin = p->n_staged, nout = p->an.n_out + p->an.n_inout, nio = p->an.n_inout, n1 = p->n1();
+    if (nin < 1 || nin_all > MAXIN || nout > MAXOUT || nio > MAXIO || n1 > MAX1D || p->ns() > MAXS)
         throw Error(SDAG_ERR_UNSUPPORTED,
                     "jit: DAG outside the sweep skeleton's limits (1.." + std::to_string(MAXIN) + " inputs, <= " +
                         std::to_string(MAXOUT) + " outputs, <= " + std::to_string(MAXIO) + " inouts, <= " +
@@ -287,7 +290,9 @@ void jit_build_candidates(Plan *p) {
     // the ring only as deep as the off-axis taps need
     int rz_off = 0;
     for (const Node &n : p->st.nodes)
-        if (n.kind == Node::Load3 && (n.off[1] != 0 || n.off[2] != 0)) rz_off = std::max(rz_off, std::abs(n.off[0]));
+        if (n.kind == Node::Load3 && (n.off[1] != 0 || n.off[2] != 0) && p->in_slot[n.ref] >= 0 &&
+            p->in_slot[n.ref] < p->n_staged)
+            rz_off = std::max(rz_off, std::abs(n.off[0]));
     struct CandQ {
         Geom g;
         bool tma;

@@ -41,6 +41,8 @@ struct Plan {
 
     // ABI mapping (per 3D formal kind_index): staged-input slot / output slot / inout slot
     std::vector<int> in_slot, out_slot, io_slot;
+    int n_staged = 0;  // inputs staged in shared memory: slots [0, n_staged); generated kernels
+                       // read the rest (#assign gmem) through L1/L2
     std::vector<const KernelDesc *> cands;  // candidate kernels (TMA first)
     std::vector<const KernelDesc *> fused;  // multi-sweep kernels for apply_iterated (tsteps > 1)
     double fcost[8] = {0};                  // f(x): relative cost of an x-sweep launch (deep tuning)

@@ -611,12 +611,25 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
     p->out_slot.assign(n3, -1);
     p->io_slot.assign(n3, -1);
     int ni = 0, no = 0, nio = 0;
+    // generated kernels honour "#assign gmem(...)": those inputs take
+    // the last slots and are read from global memory, not staged (registered
+    // kernels keep their own staging)
+    auto gmem = [&](int f) {
+        const auto &g = p->st.assign.gmem;
+        return !p->reg && std::find(g.begin(), g.end(), p->st.formal(ArgKind::Array3D, f).name) != g.end();
+    };
+    int n_in = 0, n_gm = 0;
+    for (int f = 0; f < n3; f++)
+        if (p->st.formal(ArgKind::Array3D, f).role == Role::In) (gmem(f) ? n_gm : n_in)++;
+    const bool split = n_gm > 0 && n_in > 0;  // at least one staged array
+    int ng = split ? n_in : 0;
     for (int f = 0; f < n3; f++) {
         const Role r = p->st.formal(ArgKind::Array3D, f).role;
-        if (r == Role::In) p->in_slot[f] = ni++;
+        if (r == Role::In) p->in_slot[f] = (split && gmem(f)) ? ng++ : ni++;
         if (r == Role::Out || r == Role::InOut) p->out_slot[f] = no++;
         if (r == Role::InOut) p->io_slot[f] = nio++;
     }
+    p->n_staged = ni;
     p->batch_hint = std::max(1, o.batch);
     p->tune = o.tune;
     p->fusion = o.fusion != 0;
@@ -743,9 +756,12 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
         if (pr.occupancy > 0) d << " occupancy " << pr.occupancy;
         for (auto &a : p->st.assign.gmem) d << " gmem:" << a;
         for (auto &a : p->st.assign.shmem) d << " shmem:" << a;
-        d << (p->jit_descs.empty() ? "  -- the registered sm_100a kernel keeps its measured geometry and staging "
-                                     "(force a variant, or variant \"jit\" to generate the guided one)"
-                                   : "  -- block x unroll is the first generated geometry");
+        if (p->jit_descs.empty())
+            d << "  -- the registered sm_100a kernel keeps its measured geometry and staging (force a variant, "
+                 "or variant \"jit\" to generate the guided one)";
+        else
+            d << "  -- generated kernels: block x unroll is the first geometry; " << (p->an.n_in - p->n_staged)
+              << " gmem input(s) read through L1/L2, " << p->n_staged << " staged";
     }
     if (!p->jit_descs.empty())
         d << "\n  jit body (NVRTC, sm_100a, into the sweep.cuh skeleton):\n" << jit_body_source(*p, "JitBody", p->an.radius[0]);

@@ -198,6 +198,10 @@ struct Tap {
             return __ldg(a->in[arr] + gidx + (int64_t(dz) * a->ny + dy) * a->nx + dx);
         return ring[soff[dz + RZR] + arr * PLANE_AL + base + dy * PX + dx];
     }
+    // an input assigned to global memory (#assign gmem): not staged
+    __device__ __forceinline__ double gm(int arr, int dz, int dy, int dx) const {
+        return __ldg(a->in[arr] + gidx + (int64_t(dz) * a->ny + dy) * a->nx + dx);
+    }
     __device__ __forceinline__ double io(int m) const { return a->io[m][gidx]; }
     __device__ __forceinline__ double s(int n) const { return a->s[n]; }
     __device__ __forceinline__ double s1(int arr, int off) const {
@@ -369,6 +373,9 @@ struct TapQ {
     __device__ __forceinline__ double at(int arr, int dz, int dy, int dx) const {
         if (dy == 0 && dx == 0) return qv[arr * NQ + dz + RZQ];
         return ring[soff[dz + RZR] + arr * PLANE_AL + base + dy * PX + dx];
+    }
+    __device__ __forceinline__ double gm(int arr, int dz, int dy, int dx) const {
+        return __ldg(a->in[arr] + gidx + (int64_t(dz) * a->ny + dy) * a->nx + dx);
     }
     __device__ __forceinline__ double io(int m) const { return a->io[m][gidx]; }
     __device__ __forceinline__ double s(int n) const { return a->s[n]; }
