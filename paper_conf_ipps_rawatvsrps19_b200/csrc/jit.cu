@@ -187,7 +187,7 @@ struct Compiled {
     std::string log;
 };
 
-Compiled nvrtc_build(const std::string &src, const std::vector<std::string> &names) {
+Compiled nvrtc_build(const std::string &src, const std::vector<std::string> &names, int maxrreg = 0) {
     const Nvrtc &N = nvrtc();
     nvrtcProgram prog;
     auto ck = [&](nvrtcResult r, const char *what) {
@@ -197,9 +197,11 @@ Compiled nvrtc_build(const std::string &src, const std::vector<std::string> &nam
     Compiled c;
     try {
         for (const auto &n : names) ck(N.add_name(prog, n.c_str()), "nvrtcAddNameExpression");
-        const char *opts[] = {"-arch=sm_100a", "-std=c++17", "-default-device", "--fmad=true", "-lineinfo",
-                              "--extra-device-vectorization"};
-        const nvrtcResult rc = N.compile(prog, int(sizeof opts / sizeof *opts), opts);
+        std::vector<const char *> opts = {"-arch=sm_100a", "-std=c++17", "-default-device", "--fmad=true",
+                                          "-lineinfo", "--extra-device-vectorization"};
+        const std::string rr = "--maxrregcount=" + std::to_string(maxrreg);
+        if (maxrreg > 0) opts.push_back(rr.c_str());  // occupancy t: register rationing
+        const nvrtcResult rc = N.compile(prog, int(opts.size()), opts.data());
         size_t ls = 0;
         N.log_size(prog, &ls);
         c.log.assign(ls, '\0');
@@ -246,13 +248,14 @@ struct Geom {
 // plan's DAG.  Throws UNSUPPORTED when the DAG exceeds the skeleton's limits.
 void jit_build_candidates(Plan *p) {
     using namespace dev;
-    const int nin_all = p->an.n_in, nin = p->n_staged, nout = p->an.n_out + p->an.n_inout, nio = p->an.n_inout, n1 = p->n1();
-    if (nin < 1 || nin_all > MAXIN || nout > MAXOUT || nio > MAXIO || n1 > MAX1D || p->ns() > MAXS)
+    const int nin_all = p->an.n_in, nout = p->an.n_out + p->an.n_inout, nio = p->an.n_inout, n1 = p->n1();
+    if (p->n_staged < 1 || nin_all > MAXIN || nout > MAXOUT || nio > MAXIO || n1 > MAX1D || p->ns() > MAXS)
         throw Error(SDAG_ERR_UNSUPPORTED,
                     "jit: DAG outside the sweep skeleton's limits (1.." + std::to_string(MAXIN) + " inputs, <= " +
                         std::to_string(MAXOUT) + " outputs, <= " + std::to_string(MAXIO) + " inouts, <= " +
                         std::to_string(MAX1D) + " 1D arrays, <= " + std::to_string(MAXS) + " scalars)");
     const int RZ = p->an.radius[0], RY = p->an.radius[1], RX = p->an.radius[2];
+    int nin = p->n_staged;
 
     // tile geometries, preference order (the generic skeleton's best shapes on
     // the registered DAGs: tools/perf_sweep.py); smem decides RZR
@@ -300,6 +303,45 @@ void jit_build_candidates(Plan *p) {
         std::string name;
     };
     std::vector<CandQ> cq;
+
+    // "#pragma ... occupancy t": t x 2048 threads must be resident per
+    // SM.  Registers are rationed with --maxrregcount; while shared memory still
+    // prevents it for the first geometry, the staged input with the fewest
+    // accesses is demoted to global memory (read through L1/L2, as #assign gmem),
+    // until the ring fits or one input is left staged.
+    int maxrreg = 0;
+    int nstage = nin;
+    if (pr.occupancy > 0) {
+        const Geom &g0 = geoms[0];
+        const int thr = (g0.tx / g0.ux) * (g0.ty / g0.uy);
+        const int target = std::max(thr, int(pr.occupancy * 2048.0 + 0.5));
+        maxrreg = std::max(32, std::min(255, (65536 / target) / 8 * 8));
+        const int plane_al = (((g0.tx + 2 * RX) * (g0.ty + 2 * RY) * 8 + 127) / 128) * 128 / 8;
+        auto resident = [&](int ns_in) {
+            const int smem = (2 * RZ + 1 + g0.pf) * ns_in * plane_al * 8 + (2 * RZ + 1 + g0.pf) * 8;
+            const int by_smem = smem > 0 ? (228 * 1024) / (smem + 1024) : 32;
+            return std::min(2048 / thr, by_smem) * thr;
+        };
+        std::vector<int> acc(p->n3(), 0);  // accesses per 3D formal
+        for (const Node &n : p->st.nodes)
+            if (n.kind == Node::Load3) acc[n.ref]++;
+        while (nstage > 1 && resident(nstage) < target) {
+            int victim = -1;
+            for (int f = 0; f < p->n3(); f++)
+                if (p->in_slot[f] >= 0 && p->in_slot[f] < nstage &&
+                    (victim < 0 || acc[f] < acc[victim]))
+                    victim = f;
+            // move the victim to the last staged slot, then shrink the staged range
+            const int last = nstage - 1, vs = p->in_slot[victim];
+            for (int f = 0; f < p->n3(); f++)
+                if (p->in_slot[f] == last) p->in_slot[f] = vs;
+            p->in_slot[victim] = last;
+            nstage--;
+        }
+        p->n_staged = nstage;
+        p->jit_maxrreg = maxrreg;
+        nin = nstage;
+    }
     if (RZ > 0) {
         for (const Geom &g : geoms) {
             const int px = g.tx + 2 * RX, py = g.ty + 2 * RY;
@@ -328,7 +370,8 @@ void jit_build_candidates(Plan *p) {
     if (cs.empty()) throw Error(SDAG_ERR_UNSUPPORTED, "jit: no tile geometry fits 227 KB of shared memory");
 
     std::ostringstream src;
-    src << "// generated by sdag jit.cpp for stencil '" << p->st.name << "'\n" << kSweepSrc << "\n"
+    src << "// generated by sdag jit.cpp for stencil '" << p->st.name << "'"
+        << (maxrreg ? " (--maxrregcount=" + std::to_string(maxrreg) + ")" : std::string()) << "\n" << kSweepSrc << "\n"
         << "namespace sdag {\nnamespace dev {\n";
     if (need_full) src << jit_body_source(*p, "JitBody", RZ);
     if (need_r0 && RZ > 0) src << jit_body_source(*p, "JitBodyR0", 0);
@@ -359,7 +402,7 @@ void jit_build_candidates(Plan *p) {
 
     std::lock_guard<std::mutex> lk(g_jit_mu);
     auto it = g_compiled.find(key);
-    if (it == g_compiled.end()) it = g_compiled.emplace(key, nvrtc_build(key, names)).first;
+    if (it == g_compiled.end()) it = g_compiled.emplace(key, nvrtc_build(key, names, maxrreg)).first;
     const Compiled &cc = it->second;
     p->jit_source = key;
 

@@ -759,9 +759,13 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
         if (p->jit_descs.empty())
             d << "  -- the registered sm_100a kernel keeps its measured geometry and staging (force a variant, "
                  "or variant \"jit\" to generate the guided one)";
-        else
-            d << "  -- generated kernels: block x unroll is the first geometry; " << (p->an.n_in - p->n_staged)
-              << " gmem input(s) read through L1/L2, " << p->n_staged << " staged";
+        else {
+            d << "  -- generated kernels:";
+            if (pr.block[0] > 0) d << " block x unroll is the first geometry;";
+            if (p->jit_maxrreg > 0) d << " --maxrregcount=" << p->jit_maxrreg << ";";
+            d << " " << (p->an.n_in - p->n_staged) << " gmem input(s) read through L1/L2, " << p->n_staged
+              << " staged";
+        }
     }
     if (!p->jit_descs.empty())
         d << "\n  jit body (NVRTC, sm_100a, into the sweep.cuh skeleton):\n" << jit_body_source(*p, "JitBody", p->an.radius[0]);
