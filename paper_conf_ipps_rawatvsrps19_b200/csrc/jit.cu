@@ -401,14 +401,15 @@ void jit_build_candidates(Plan *p) {
     const std::string key = src.str();
 
     std::lock_guard<std::mutex> lk(g_jit_mu);
-    auto it = g_compiled.find(key);
-    if (it == g_compiled.end()) it = g_compiled.emplace(key, nvrtc_build(key, names, maxrreg)).first;
-    const Compiled &cc = it->second;
-    p->jit_source = key;
-
-    std::vector<CUfunction> fns(cs.size(), nullptr);
-    if (!p->host_only) {
-        auto mk = std::make_pair(key, p->device);
+    // compile (cached by source and register cap) and load on the plan's device
+    auto build = [&](int cap) {
+        const std::string ck = cap ? key + "// --maxrregcount=" + std::to_string(cap) + "\n" : key;
+        auto it = g_compiled.find(ck);
+        if (it == g_compiled.end()) it = g_compiled.emplace(ck, nvrtc_build(key, names, cap)).first;
+        const Compiled &cc = it->second;
+        std::vector<CUfunction> fns(names.size(), nullptr);
+        if (p->host_only) return fns;
+        auto mk = std::make_pair(ck, p->device);
         auto mt = g_mods.find(mk);
         if (mt == g_mods.end()) {
             int prev = -1;
@@ -430,8 +431,10 @@ void jit_build_candidates(Plan *p) {
             check_cu(r, "jit: cuModuleLoadData/cuModuleGetFunction");
             mt = g_mods.emplace(mk, m).first;
         }
-        fns = mt->second.fns;
-    }
+        return mt->second.fns;
+    };
+    p->jit_source = key;
+    std::vector<CUfunction> fns = build(maxrreg);
     for (size_t q = 0; q < cs.size(); q++) {
         const Cand &c = cs[q];
         auto d = std::make_unique<KernelDesc>();
@@ -483,6 +486,31 @@ void jit_build_candidates(Plan *p) {
         d->rzr = rz_off;
         d->prio = -10 + int(q / 2) + (c.tma ? 0 : 100);  // preferred: 1.35x (lap25), 1.1x (27-pt) over the ring-only skeleton
         p->jit_descs.push_back(std::move(d));
+    }
+
+    // register-cap stepping: with tune=1 the TMA candidates are
+    // also compiled at 128 and 64 registers per thread; the spill-free ones
+    // (no local memory) join the measured candidates as "<variant>_rr<cap>"
+    if (p->tune && !p->host_only && maxrreg == 0) {
+        using AttrT = decltype(&cuFuncGetAttribute);
+        const size_t base = p->jit_descs.size();
+        for (int cap : {128, 64}) {
+            const std::vector<CUfunction> cf = build(cap);
+            for (size_t q = 0; q < base; q++) {
+                const KernelDesc &k0 = *p->jit_descs[q];
+                if (!k0.tma) continue;
+                const size_t fi = q;  // descriptors were created in name order
+                int local = 0;
+                check_cu(drv<AttrT>("cuFuncGetAttribute")(&local, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, cf[fi]),
+                         "jit: cuFuncGetAttribute");
+                if (local > 0) continue;  // spills: not explored
+                auto d = std::make_unique<KernelDesc>(k0);
+                d->variant += "_rr" + std::to_string(cap);
+                d->cufn = cf[fi];
+                d->prio += 50;
+                p->jit_descs.push_back(std::move(d));
+            }
+        }
     }
 }
 

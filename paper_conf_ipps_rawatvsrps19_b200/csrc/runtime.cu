@@ -877,7 +877,7 @@ static void time_candidates(Plan *p) {
         check_cuda(cudaEventCreate(&e1), "event");
         float best = 1e30f;
         int bestq = 0;
-        for (size_t q = 0; q < p->cands.size() && q < 16; q++) {
+        for (size_t q = 0; q < p->cands.size() && q < 32; q++) {
             const KernelDesc &k = *p->cands[q];
             if (!k.tma && p->dims[2] % 2 == 0) continue;  // LSU twins only matter for odd nx
             plan_launch(p, k, b3.data(), b1.data(), s.data(), p->batch_hint, 0, p->dims[0], 0);
