@@ -41,7 +41,9 @@ struct Plan {
 
     // ABI mapping (per 3D formal kind_index): staged-input slot / output slot / inout slot
     std::vector<int> in_slot, out_slot, io_slot;
-    int jit_maxrreg = 0;  // --maxrregcount of the generated kernels (occupancy t), 0 = none
+    int jit_maxrreg = 0;
+    int zchunk_tuned = 0;   // z-chunk length chosen by tune=1 (0 = the occupancy model's)
+    int tuned_timed = 0;    // candidates timed by the hierarchical tuner  // --maxrregcount of the generated kernels (occupancy t), 0 = none
     int n_staged = 0;  // inputs staged in shared memory: slots [0, n_staged); generated kernels
                        // read the rest (#assign gmem) through L1/L2
     std::vector<const KernelDesc *> cands;  // candidate kernels (TMA first)

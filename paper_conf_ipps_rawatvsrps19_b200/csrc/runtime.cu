@@ -5,6 +5,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <set>
 #include <fstream>
 #include <functional>
 #include <sstream>
@@ -182,6 +183,11 @@ static void geometry(const Plan *p, const KernelDesc &k, int batch, int64_t klo,
             best = cost;
             bestn = n;
         }
+    }
+    // tuned z-chunk length (tune=1, step 3) for launches over the plan's own z-range
+    if (p->zchunk_tuned > 0 && klo == p->lo[0] && khi == p->hi[0]) {
+        const int64_t zc = std::min<int64_t>(nzi, p->zchunk_tuned);
+        bestn = int(std::min<int64_t>(maxn, (nzi + zc - 1) / zc));
     }
     // debug/ablation override of the chunk count (tools/chunk_sweep.py)
     if (const char *e = std::getenv("SDAG_NCHUNK")) {
@@ -737,7 +743,10 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
     const KernelDesc &k = p->kernel();
     d << "\n  variant " << k.variant << " (" << k.threads << " threads, " << k.smem << " B smem, ring "
       << (2 * k.rzr + 1 + k.pf) << " planes)"
-      << (p->tune ? (p->tune_cached ? "  [tuned, from $SDAG_TUNE_CACHE]" : "  [tuned]") : "  [heuristic]")
+      << (p->tune ? (p->tune_cached ? "  [tuned, from $SDAG_TUNE_CACHE]"
+                                    : "  [tuned: " + std::to_string(p->tuned_timed) + " candidates timed]")
+                  : "  [heuristic]")
+      << (p->zchunk_tuned > 0 ? "  z-chunk " + std::to_string(p->zchunk_tuned) + " planes (tuned)" : "")
       << "\n  candidates:";
     for (auto *c : p->cands) d << " " << c->variant;
     if (!p->fused.empty()) {
@@ -827,6 +836,7 @@ static bool tune_cache_load(Plan *p) {
     p->chosen = chosen;
     for (int x = 1; x < 8; x++) p->fcost[x] = f[x];
     if (!fused.empty()) p->fused = fused;
+    if (col.size() > 4 && !col[4].empty()) p->zchunk_tuned = std::max(0, std::atoi(col[4].c_str()));
     return true;
 }
 
@@ -841,7 +851,7 @@ static void tune_cache_store(const Plan *p) {
     for (int x = 1; x < 8; x++) out << (x > 1 ? " " : "") << p->fcost[x];
     out << "\t";
     for (size_t q = 0; q < p->fused.size(); q++) out << (q ? "," : "") << p->fused[q]->variant;
-    out << "\n";
+    out << "\t" << p->zchunk_tuned << "\n";
 }
 
 // Hierarchical autotuning, lite: time every candidate geometry on
@@ -875,11 +885,7 @@ static void time_candidates(Plan *p) {
         cudaEvent_t e0, e1;
         check_cuda(cudaEventCreate(&e0), "event");
         check_cuda(cudaEventCreate(&e1), "event");
-        float best = 1e30f;
-        int bestq = 0;
-        for (size_t q = 0; q < p->cands.size() && q < 32; q++) {
-            const KernelDesc &k = *p->cands[q];
-            if (!k.tma && p->dims[2] % 2 == 0) continue;  // LSU twins only matter for odd nx
+        auto time_k = [&](const KernelDesc &k) {
             plan_launch(p, k, b3.data(), b1.data(), s.data(), p->batch_hint, 0, p->dims[0], 0);
             check_cuda(cudaEventRecord(e0, 0), "event");
             for (int r = 0; r < 3; r++)
@@ -888,12 +894,65 @@ static void time_candidates(Plan *p) {
             check_cuda(cudaEventSynchronize(e1), "event sync");
             float ms = 0;
             check_cuda(cudaEventElapsedTime(&ms, e0, e1), "event time");
-            if (ms < best) {
-                best = ms;
+            return ms;
+        };
+        // Hierarchical autotuning.  Step 1, the high-impact
+        // choices: one representative (the preferred variant) per thread-block
+        // geometry (tile, unroll, loader).  Step 2: every other variant of the
+        // three fastest geometries (prefetch depth, queue/unroll forms, register
+        // caps).  Step 3, concurrent streaming: the z-chunk length of
+        // the winner, around the occupancy model's pick.
+        auto geo = [](const KernelDesc *k) {
+            return std::to_string(k->tx) + "x" + std::to_string(k->ty) + "u" + std::to_string(k->ux) + "x" +
+                   std::to_string(k->uy) + (k->tma ? "t" : "l");
+        };
+        std::vector<float> tq(p->cands.size(), -1.0f);
+        std::vector<std::pair<float, std::string>> groups;
+        std::set<std::string> seen;
+        for (size_t q = 0; q < p->cands.size() && q < 64; q++) {
+            const KernelDesc &k = *p->cands[q];
+            if (!k.tma && p->dims[2] % 2 == 0) continue;  // LSU twins only matter for odd nx
+            if (!seen.insert(geo(&k)).second) continue;
+            tq[q] = time_k(k);
+            groups.push_back({tq[q], geo(&k)});
+        }
+        std::stable_sort(groups.begin(), groups.end(), [](auto &a, auto &b) { return a.first < b.first; });
+        std::set<std::string> top;
+        for (size_t g = 0; g < groups.size() && g < 3; g++) top.insert(groups[g].second);
+        for (size_t q = 0; q < p->cands.size() && q < 64; q++) {
+            const KernelDesc &k = *p->cands[q];
+            if (tq[q] >= 0 || !top.count(geo(&k))) continue;
+            if (!k.tma && p->dims[2] % 2 == 0) continue;
+            tq[q] = time_k(k);
+        }
+        float best = 1e30f;
+        int bestq = 0;
+        for (size_t q = 0; q < tq.size(); q++)
+            if (tq[q] >= 0 && tq[q] < best) {
+                best = tq[q];
                 bestq = int(q);
             }
-        }
         p->chosen = bestq;
+        p->tuned_timed = int(std::count_if(tq.begin(), tq.end(), [](float v) { return v >= 0; }));
+        {
+            const KernelDesc &k = *p->cands[bestq];
+            Launch L0;
+            int64_t zlo[3] = {p->lo[0], p->lo[1], p->lo[2]}, zhi[3] = {p->hi[0], p->hi[1], p->hi[2]};
+            geometry(p, k, p->batch_hint, p->lo[0], p->hi[0], zlo, zhi, L0);
+            const int64_t nzi = p->hi[0] - p->lo[0];
+            int best_zc = 0;
+            for (double f : {0.25, 0.5, 2.0, 4.0}) {
+                const int64_t zc = std::max<int64_t>(1, std::min<int64_t>(nzi, int64_t(L0.zchunk * f + 0.5)));
+                if (zc == L0.zchunk) continue;
+                p->zchunk_tuned = int(zc);
+                const float ms = time_k(k);
+                if (ms < 0.98f * best) {  // a clear win over the model's pick
+                    best = ms;
+                    best_zc = int(zc);
+                }
+            }
+            p->zchunk_tuned = best_zc;
+        }
         // deep tuning: measure f(x) of every fused x-sweep kernel
         // relative to the chosen single sweep, fastest fused kernel per x first
         if (!p->fused.empty() && p->dims[2] % 2 == 0 && best < 1e29f) {

@@ -72,7 +72,7 @@ def test_tuned_plan_is_correct():
     dims = (24, 40, 72)
     case = make_case("lap25", dims)
     g, plan = run_gpu("lap25", dims, case, tune=True)
-    assert "[tuned]" in plan.describe()
+    assert "[tuned: " in plan.describe()  # hierarchical: geometries, then their variants, then z-chunks
     check("lap25", dims, g, case)
 
 
@@ -83,7 +83,7 @@ def test_persistent_tune_cache(tmp_path, monkeypatch):
     monkeypatch.setenv("SDAG_TUNE_CACHE", str(path))
     dims = (40, 48, 64)
     p1 = sdag.Plan(sdag.spec_text("smooth27"), dims, tune=True)
-    assert "[tuned]" in p1.describe()
+    assert "[tuned: " in p1.describe()
     lines = path.read_text().splitlines()
     assert len(lines) == 1 and p1.info["variant"] in lines[0]
     p2 = sdag.Plan(sdag.spec_text("smooth27"), dims, tune=True)
@@ -93,6 +93,9 @@ def test_persistent_tune_cache(tmp_path, monkeypatch):
     f1 = [ln for ln in p1.describe().splitlines() if "f(1)=" in ln]
     f2 = [ln for ln in p2.describe().splitlines() if "f(1)=" in ln]
     assert [x.split(":", 1)[1] for x in f1] == [x.split(":", 1)[1] for x in f2]
+    z1 = [w for w in p1.describe().split("  ") if w.startswith("z-chunk")]
+    z2 = [w for w in p2.describe().split("  ") if w.startswith("z-chunk")]
+    assert z1 == z2  # the tuned z-chunk length is restored too
     case = make_case("smooth27", dims)
     g1, _ = run_gpu("smooth27", dims, case, variant=p1.info["variant"])
     check("smooth27", dims, g1, case)
