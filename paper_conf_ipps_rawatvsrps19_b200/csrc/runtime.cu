@@ -184,8 +184,9 @@ static void geometry(const Plan *p, const KernelDesc &k, int batch, int64_t klo,
             bestn = n;
         }
     }
-    // tuned z-chunk length (tune=1, step 3) for launches over the plan's own z-range
-    if (p->zchunk_tuned > 0 && klo == p->lo[0] && khi == p->hi[0]) {
+    // tuned z-chunk length (tune=1, step 3): launches of the tuned kernel over the
+    // plan's own z-range
+    if (p->zchunk_tuned > 0 && klo == p->lo[0] && khi == p->hi[0] && p->chosen >= 0 && &k == &p->kernel()) {
         const int64_t zc = std::min<int64_t>(nzi, p->zchunk_tuned);
         bestn = int(std::min<int64_t>(maxn, (nzi + zc - 1) / zc));
     }

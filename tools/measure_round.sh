@@ -7,7 +7,7 @@ mkdir -p gpurun_out/meas
 M=gpurun_out/meas
 timeout 1500 python -m pytest tests -q -m gpu --timeout 900 > $M/pytest_gpu.log 2>&1; echo "exit $?" >> $M/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke(); print('smoke ok')" > $M/smoke.log 2>&1
-timeout 600 python bench.py > $M/bench_lap25.json 2> $M/bench_lap25.err
+timeout 600 python bench.py > $M/bench_lap25.json 2> $M/bench_lap25.err   # headline: heuristic plan
 for c in jacobi7 hypterm rhs4center smooth27; do
   timeout 600 python bench.py --config $c > $M/bench_$c.json 2> $M/bench_$c.err
 done
