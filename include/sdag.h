@@ -200,7 +200,7 @@ sdag_status sdag_apply_iterated(sdag_plan plan, double *buf0, double *buf1, int3
  * copies every 3D input/inout and 1D array host->device into a plan-owned
  * workspace, runs one sweep, copies the interior of every output/inout
  * device->host (the host ring is not written), and synchronises `stream`.
- * Pipelined over z-chunks of the output (<= 16 chunks of >= max(8, 2R_z)
+ * Pipelined over z-chunks of the output (<= 64 chunks of >= max(10, 2R_z)
  * planes): the H2D of chunk c+1 (plan-owned copy stream), the sweep of chunk c
  * (`stream`) and the D2H of chunk c-1 (second copy stream) overlap; every
  * input plane crosses the link once.  Calls on one plan are serialised.

@@ -489,9 +489,14 @@ void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int
     }
     const int64_t R = p->an.radius[0];
     const int64_t zlo = p->lo[0], zhi = p->hi[0];
-    // chunks of >= 8 planes (and >= 2R_z so the halo share stays small), at most 16
+    // chunks of >= 10 planes (and >= 2R_z so the halo share stays small), at
+    // most 64: the pipeline fill (first upload) and drain (last download) are
+    // one chunk each; measured on B200 at 512^3 (tools/e2e_probe.py): 16 chunks
+    // 27.8 ms, 32: 26.2, 48: 25.1, 63 (8 planes): 26.2
     const int64_t nzi = std::max<int64_t>(0, zhi - zlo);
-    const int64_t nch = std::max<int64_t>(1, std::min<int64_t>(16, nzi / std::max<int64_t>(8, 2 * R)));
+    int64_t maxch = 64;
+    if (const char *e = std::getenv("SDAG_HOST_CHUNKS")) maxch = std::max(1, std::atoi(e));  // ablation
+    const int64_t nch = std::max<int64_t>(1, std::min<int64_t>(maxch, nzi / std::max<int64_t>(10, 2 * R)));
     const int64_t zc = nzi > 0 ? (nzi + nch - 1) / nch : 0;
 
     std::vector<double *> d3(n3);
