@@ -388,8 +388,8 @@ def main():
     ap.add_argument("--config", default="lap25", choices=list(CONFIGS),
                     help="lap25 = the headline line; the others record the remaining BASELINE stencils (N=1)")
     ap.add_argument("--halo", default=None, choices=["nccl", "p2p"],
-                    help="with --config smooth27: the z-slab run of config 5 (BASELINE's multi-GPU workload) "
-                         "with this halo path")
+                    help="z-slab halo path (default nccl); with --config smooth27: the z-slab run of config 5 "
+                         "(BASELINE's multi-GPU workload)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
@@ -405,18 +405,23 @@ def main():
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = 0 if os.environ.get("SDAG_BENCH_SAME_DEVICE") else int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
+    p2p = args.halo == "p2p"
     dist = None
     if world > 1:
         import torch.distributed as tdist
-        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if p2p:  # host plumbing only (IPC handles, barriers, the timing reduce)
+            tdist.init_process_group("gloo")
+        else:
+            tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
         dist = tdist
+    red_dev = "cpu" if p2p else "cuda"
     name = "lap25"
     spec = sdag.spec_text(name)
     ldims = CONFIGS[name][1]
     gdims = (ldims[0] * world, ldims[1], ldims[2])
-    use_dist = world > 1 or args.force_dist
+    use_dist = world > 1 or args.force_dist or args.halo == "p2p"
     ins, sc = synth.lap25_inputs(ldims, cfg="cfg2") if not use_dist else (None, dict(synth.LAP25_COEFS))
     c = [sc[k] for k in ("c0", "c1", "c2", "c3", "c4")]
     stream = torch.cuda.current_stream()
@@ -433,17 +438,35 @@ def main():
         def step():
             plan.apply(arrays, scalars=c, stream=stream)
     else:
-        uid = [sdag.nccl_unique_id() if rank == 0 else None]
-        if dist:
-            dist.broadcast_object_list(uid, src=0)
-        comm = sdag.nccl_comm_create(uid[0], world, rank, local)
+        comm = None
+        if not p2p:
+            uid = [sdag.nccl_unique_id() if rank == 0 else None]
+            if dist:
+                dist.broadcast_object_list(uid, src=0)
+            comm = sdag.nccl_comm_create(uid[0], world, rank, local)
         dd = sdag.Dist(spec, gdims, rank, world, comm=comm, tune=args.tune, variant=args.variant)
         (nza, ny, nx), g0 = dd.layout()
         part = sdag.slab_partition(gdims[0], 4, world, rank)
         # this rank's slab of the global synthetic input, regenerated from the counter-based generator
         full = synth.uniform((nza, ny, nx), -1.0, 1.0, "cfg2-slab", rank)
-        dA = torch.from_numpy(full).cuda()
-        dB = torch.zeros((nza, ny, nx), dtype=torch.float64, device="cuda")
+        if p2p:
+            # --halo p2p: library-owned slab buffers; the input's ghost planes are
+            # pushed over NVLink by the neighbours and flag-ordered (one sweep =
+            # sdag_dist_p2p_apply_iterated with T = 1), no NCCL
+            dA, dB = dd.p2p_alloc()
+            dA.copy_(torch.from_numpy(full))
+            dB.zero_()
+            torch.cuda.synchronize()
+            if dist:
+                hs = [None] * world
+                dist.all_gather_object(hs, dd.p2p_handle())
+                if rank > 0:
+                    dd.p2p_attach(0, hs[rank - 1])
+                if rank < world - 1:
+                    dd.p2p_attach(1, hs[rank + 1])
+        else:
+            dA = torch.from_numpy(full).cuda()
+            dB = torch.zeros((nza, ny, nx), dtype=torch.float64, device="cuda")
         arrays = [dB, dA]
         plan = dd.plan
         info = plan.info
@@ -451,7 +474,10 @@ def main():
         comm_stream = torch.cuda.Stream()
 
         def step():
-            dd.apply(arrays, scalars=c, stream=stream, comm_stream=comm_stream)
+            if p2p:
+                dd.p2p_apply_iterated(1, scalars=c, stream=stream)
+            else:
+                dd.apply(arrays, scalars=c, stream=stream, comm_stream=comm_stream)
 
     flops_pt = info["flops_per_point"]
     for _ in range(args.warmup):
@@ -470,8 +496,8 @@ def main():
         torch.cuda.synchronize()
     launches = sdag.launch_count() - l0
     ms = e0.elapsed_time(e1)
-    ms_t = torch.tensor([ms], dtype=torch.float64, device="cuda")
-    pts_t = torch.tensor([float(pts_rank)], dtype=torch.float64, device="cuda")
+    ms_t = torch.tensor([ms], dtype=torch.float64, device=red_dev)
+    pts_t = torch.tensor([float(pts_rank)], dtype=torch.float64, device=red_dev)
     if dist:
         dist.barrier()
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
@@ -525,12 +551,12 @@ def main():
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             dA.copy_(hA, non_blocking=True)
-            dd.apply(arrays, scalars=c, stream=stream, comm_stream=comm_stream)
+            step()
             hB.copy_(dB[z0:z0 + nown], non_blocking=True)
             torch.cuda.synchronize()
             if it:
                 ee.append(time.perf_counter() - t0)
-        t_loc = torch.tensor([statistics.median(ee)], dtype=torch.float64, device="cuda")
+        t_loc = torch.tensor([statistics.median(ee)], dtype=torch.float64, device=red_dev)
         if dist:
             dist.all_reduce(t_loc, op=dist.ReduceOp.MAX)
         t_e2e = float(t_loc.item())
@@ -549,6 +575,7 @@ def main():
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": CONFIGS[name][2], "stencil": name, "grid_per_gpu": list(ldims),
                        "global_grid": list(gdims), "decomposition": f"z-slabs x{world}" if use_dist else "none",
+                       "halo": ("p2p" if p2p else "nccl") if use_dist else None,
                        "variant": info["variant"], "flops_per_point": flops_pt,
                        "bytes_per_point": info["bytes_per_point"],
                        "l2": "input 1 GiB/GPU > 126 MB L2 (no flush needed)"},
