@@ -354,6 +354,18 @@ enum { SDAG_FISSION_MAXFUSE = 0, SDAG_FISSION_TRIVIAL = 1 };
  * INVALID_ARG is returned when buf is non-null and too small.  Parse and
  * semantic errors as sdag_plan_create.  Host only. */
 sdag_status sdag_spec_fission(const char *spec, int32_t kind, char *buf, int64_t cap, int64_t *len);
+/* The reverse direction for a multi-stencil program (Fig 3c form): maxfuse with
+ * recomputation -- ONE stencil in which every read of an array an earlier stage
+ * wrote is replaced by that stage's expression at the read's offset
+ * (temporaries inlined), so intermediates never go through memory.  The fused
+ * stencil's radius is the composed one; on its interior every written value is
+ * computed by the same operations as in the staged program.  Its formals are
+ * the program's declared arguments (declaration order).  keep_intermediates = 0:
+ * arrays read by a later stage are not written (only the sinks).  UNSUPPORTED
+ * when a written array is also read at an offset before any stage writes it.
+ * Buffer convention as sdag_spec_fission.  Host only. */
+sdag_status sdag_program_fuse(const char *program, int32_t keep_intermediates, char *buf, int64_t cap,
+                              int64_t *len);
 
 /* ------------------------------------------------------------------------
  * Profile-guided classification (paper Section IV)

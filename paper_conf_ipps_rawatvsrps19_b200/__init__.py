@@ -21,7 +21,7 @@ import os
 from . import _capi
 from ._capi import PlanInfo, PlanOpts, SDAG_DEVICE_CURRENT, SDAG_DEVICE_NONE
 
-__all__ = ["Plan", "Program", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "slab_partition2", "slab_halo2", "fission", "nccl_unique_id",
+__all__ = ["Plan", "Program", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "slab_partition2", "slab_halo2", "fission", "fuse_program", "nccl_unique_id",
            "nccl_comm_create", "nccl_comm_destroy", "launch_count", "fp64_peak", "version", "SPEC_DIR"]
 
 SPEC_DIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "specs")
@@ -463,6 +463,17 @@ def fission(spec: str, kind: str = "trivial") -> str:
     _check(L.sdag_spec_fission(spec.encode(), k, None, 0, ctypes.byref(n)))
     buf = ctypes.create_string_buffer(n.value + 1)
     _check(L.sdag_spec_fission(spec.encode(), k, buf, n.value + 1, ctypes.byref(n)))
+    return buf.value.decode()
+
+
+def fuse_program(program: str, keep_intermediates: bool = True) -> str:
+    """maxfuse of a multi-stencil program with recomputation (sdag_program_fuse):
+    one stencil; intermediates inlined at their read offsets"""
+    L = _capi.lib()
+    n = ctypes.c_int64()
+    _check(L.sdag_program_fuse(program.encode(), int(keep_intermediates), None, 0, ctypes.byref(n)))
+    buf = ctypes.create_string_buffer(n.value + 1)
+    _check(L.sdag_program_fuse(program.encode(), int(keep_intermediates), buf, n.value + 1, ctypes.byref(n)))
     return buf.value.decode()
 
 

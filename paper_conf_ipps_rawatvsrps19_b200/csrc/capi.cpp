@@ -340,6 +340,18 @@ sdag_status sdag_spec_fission(const char *spec, int32_t kind, char *buf, int64_t
     });
 }
 
+sdag_status sdag_program_fuse(const char *program, int32_t keep, char *buf, int64_t cap, int64_t *len) {
+    return guard([&] {
+        if (!program || !len) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null argument");
+        const std::string t = sdag::fuse_program(program, keep);
+        *len = int64_t(t.size());
+        if (buf) {
+            if (cap <= *len) throw sdag::Error(SDAG_ERR_INVALID_ARG, "buffer too small");
+            std::memcpy(buf, t.c_str(), t.size() + 1);
+        }
+    });
+}
+
 sdag_status sdag_plan_profile(sdag_plan plan, void *const *a3, int32_t n3, const double *const *a1, int32_t n1,
                               const double *s, int32_t ns, double peak_hbm_gbs, double peak_fp64_tflops,
                               sdag_stream stream, sdag_profile *out) {

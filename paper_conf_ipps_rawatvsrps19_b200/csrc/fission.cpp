@@ -249,3 +249,162 @@ std::string emit_fission(const std::string &spec, int kind) {
 }
 
 }  // namespace sdag
+
+// ---------------------------------------------------------------------------
+// maxfuse of a multi-stencil program (Section VI-B "maxfuse", P:1505-1512,
+// with the recomputation the paper weighs against fusion): the
+// stages are fused into ONE stencil.  A read of an array that an earlier stage
+// wrote is replaced by that stage's expression for it, evaluated at the
+// read's offset (temporaries inlined, shifted), so the intermediate never goes
+// through memory and is recomputed once per use.  The fused stencil's radius
+// is the composed one (e.g. 1 + 1 for a Laplacian of a Laplacian) and it
+// writes every program output on ITS interior: there each value is computed
+// by exactly the operations the staged program performs.
+// ---------------------------------------------------------------------------
+
+namespace sdag {
+
+namespace {
+
+struct Fuser {
+    const ProgramIR &ir;
+    std::vector<std::string> iters;
+    std::vector<int> writer_end;  // per program arg: not used
+
+    const std::string &argname(int s, int formal_pos) const { return ir.args[ir.map[s][formal_pos]].name; }
+    int arg_of(int s, ArgKind k, int kind_index) const {
+        const Stencil &st = ir.stages[s];
+        for (size_t q = 0; q < st.formals.size(); q++)
+            if (st.formals[q].kind == k && st.formals[q].kind_index == kind_index) return ir.map[s][q];
+        throw Error(SDAG_ERR_INVALID_ARG, "fuse: formal not bound");
+    }
+    std::string idx(int axis, int off) const {
+        const std::string &it = iters[axis];
+        if (off == 0) return it;
+        return it + (off > 0 ? "+" : "-") + std::to_string(std::abs(off));
+    }
+    // last statement < q of stage s writing 3D arg a (or -1)
+    int last_write(int s, int a, int q) const {
+        const Stencil &st = ir.stages[s];
+        for (int r = q - 1; r >= 0; r--)
+            if (st.stmts[r].to_array && arg_of(s, ArgKind::Array3D, st.stmts[r].target) == a) return r;
+        return -1;
+    }
+    int last_temp(int s, int t, int q) const {
+        const Stencil &st = ir.stages[s];
+        for (int r = q - 1; r >= 0; r--)
+            if (!st.stmts[r].to_array && st.stmts[r].target == t) return r;
+        return -1;
+    }
+    // value of 3D arg a as stage s (before statement q) sees it, at shift d
+    std::string value(int s, int q, int a, const int d[3], const std::vector<bool> &fused_writes) const {
+        const int w = last_write(s, a, q);
+        if (w >= 0) return "(" + expr(s, w, ir.stages[s].stmts[w].expr, d, fused_writes) + ")";
+        for (int e = s - 1; e >= 0; e--) {  // the last earlier stage that wrote a
+            const int we = last_write(e, a, int(ir.stages[e].stmts.size()));
+            if (we >= 0) return "(" + expr(e, we, ir.stages[e].stmts[we].expr, d, fused_writes) + ")";
+        }
+        // a program input (or an output's initial contents)
+        if (fused_writes[a] && (d[0] || d[1] || d[2]))
+            throw Error(SDAG_ERR_UNSUPPORTED, "fuse: array '" + ir.args[a].name +
+                                                  "' is read at an offset before any stage writes it and is also "
+                                                  "written by the fused stencil");
+        std::string s3 = ir.args[a].name;
+        for (int ax = 0; ax < 3; ax++) s3 += "[" + idx(ax, d[ax]) + "]";
+        return s3;
+    }
+    std::string expr(int s, int q, int n, const int d[3], const std::vector<bool> &fw) const {
+        const Stencil &st = ir.stages[s];
+        const Node &x = st.nodes[n];
+        switch (x.kind) {
+            case Node::Num: return num(x.value);
+            case Node::Scalar: return ir.args[arg_of(s, ArgKind::Scalar, x.ref)].name;
+            case Node::Temp: {
+                const int r = last_temp(s, x.ref, q);
+                if (r < 0) throw Error(SDAG_ERR_SEMANTIC, "fuse: temporary read before assignment");
+                return "(" + expr(s, r, st.stmts[r].expr, d, fw) + ")";
+            }
+            case Node::Load3: {
+                const int dd[3] = {x.off[0] + d[0], x.off[1] + d[1], x.off[2] + d[2]};
+                return value(s, q, arg_of(s, ArgKind::Array3D, x.ref), dd, fw);
+            }
+            case Node::Load1: {
+                const int a = arg_of(s, ArgKind::Array1D, x.ref);
+                const int ax = ir.args[a].axis;
+                return ir.args[a].name + "[" + idx(ax, x.off[0] + (ax >= 0 ? d[ax] : 0)) + "]";
+            }
+            case Node::Neg: return "(-" + expr(s, q, x.a, d, fw) + ")";
+            case Node::Add: return "(" + expr(s, q, x.a, d, fw) + " + " + expr(s, q, x.b, d, fw) + ")";
+            case Node::Sub: return "(" + expr(s, q, x.a, d, fw) + " - " + expr(s, q, x.b, d, fw) + ")";
+            case Node::Mul: return "(" + expr(s, q, x.a, d, fw) + " * " + expr(s, q, x.b, d, fw) + ")";
+            case Node::Div: return "(" + expr(s, q, x.a, d, fw) + " / " + expr(s, q, x.b, d, fw) + ")";
+        }
+        throw Error(SDAG_ERR_INVALID_ARG, "fuse: unknown node");
+    }
+};
+
+}  // namespace
+
+std::string fuse_program(const std::string &text, int keep_intermediates) {
+    const ProgramIR ir = parse_program(text);
+    if (ir.stages.empty()) throw Error(SDAG_ERR_INVALID_ARG, "fuse: empty program");
+    for (const Stencil &st : ir.stages) {
+        (void)analyse(st);
+        if (st.iterators != ir.stages[0].iterators || st.iterators.size() != 3)
+            throw Error(SDAG_ERR_UNSUPPORTED, "fuse: stages must share three iterators");
+    }
+    Fuser F{ir, ir.stages[0].iterators, {}};
+    const int na = int(ir.args.size());
+    // arrays some stage writes, in order of their last write; read later?
+    std::vector<bool> written(na, false), read_later(na, false);
+    std::vector<std::pair<int, int>> last;  // (stage, arg) of each written arg's final write
+    for (size_t s = 0; s < ir.stages.size(); s++) {
+        const Stencil &st = ir.stages[s];
+        for (const Statement &w : st.stmts)
+            if (w.to_array) written[F.arg_of(int(s), ArgKind::Array3D, w.target)] = true;
+    }
+    for (size_t s = 0; s < ir.stages.size(); s++) {
+        const Stencil &st = ir.stages[s];
+        for (const Node &n : st.nodes)
+            if (n.kind == Node::Load3) {
+                const int a = F.arg_of(int(s), ArgKind::Array3D, n.ref);
+                for (size_t e = 0; e < s; e++)
+                    if (F.last_write(int(e), a, int(ir.stages[e].stmts.size())) >= 0) read_later[a] = true;
+            }
+    }
+    std::vector<bool> fw(na, false);  // arrays the fused stencil writes
+    for (int a = 0; a < na; a++) fw[a] = written[a] && (keep_intermediates || !read_later[a]);
+    std::ostringstream o;
+    o << "iterator " << F.iters[0] << ", " << F.iters[1] << ", " << F.iters[2] << ";\ndouble";
+    bool first = true;
+    for (const ProgramArg &a : ir.args) {
+        o << (first ? " " : ", ") << a.name;
+        if (a.kind == ArgKind::Array3D) o << "[64,64,64]";
+        if (a.kind == ArgKind::Array1D) o << "[64]";
+        first = false;
+    }
+    o << ";\nstencil fused (";
+    for (int a = 0; a < na; a++) o << (a ? ", " : "") << ir.args[a].name;
+    o << ") {\n";
+    const int zero[3] = {0, 0, 0};
+    int nout = 0;
+    for (int a = 0; a < na; a++) {
+        if (!fw[a]) continue;
+        // the final value: the last stage writing a, after all its statements
+        for (int s = int(ir.stages.size()) - 1; s >= 0; s--) {
+            const int w = F.last_write(s, a, int(ir.stages[s].stmts.size()));
+            if (w < 0) continue;
+            o << "    " << ir.args[a].name << "[" << F.iters[0] << "][" << F.iters[1] << "][" << F.iters[2]
+              << "] = " << F.expr(s, w, ir.stages[s].stmts[w].expr, zero, fw) << ";\n";
+            nout++;
+            break;
+        }
+    }
+    if (!nout) throw Error(SDAG_ERR_SEMANTIC, "fuse: the program writes no array");
+    o << "}\nfused (";
+    for (int a = 0; a < na; a++) o << (a ? ", " : "") << ir.args[a].name;
+    o << ");\n";
+    return o.str();
+}
+
+}  // namespace sdag

@@ -127,6 +127,9 @@ Analysis analyse(const Stencil &st);
 // fission versions of a single-stage spec as DSL program text (fission.cpp):
 // kind 0 maxfuse, 1 trivial-fission
 std::string emit_fission(const std::string &spec, int kind);
+// maxfuse of a multi-stencil program with recomputation (fission.cpp): one
+// stencil; keep_intermediates = 0 writes only arrays no later stage reads
+std::string fuse_program(const std::string &text, int keep_intermediates);
 // canonical, name-free serialisation used to match registered DAGs
 std::string canonical_form(const Stencil &st);
 
