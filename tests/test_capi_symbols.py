@@ -1,4 +1,5 @@
 """The C-ABI library loads without a GPU and exports every entry point that
+import pytest
 include/sdag.h declares (no compute calls)."""
 import os
 import re
@@ -49,3 +50,28 @@ def test_profile_struct_layout():
     from paper_conf_ipps_rawatvsrps19_b200 import _capi
     assert _capi.Profile.hints.offset == 96 + 11 * 8 + 5 * 4
     assert ctypes.sizeof(_capi.Profile) == 96 + 11 * 8 + 5 * 4 + 1024 + 4  # padded to 8
+
+
+def test_plain_c_client(tmp_path):
+    """the boundary is a C ABI: examples/c_api_host.c (no Python, no torch) builds
+    against include/sdag.h + libsdag.so, plans Listing 1 host-only, reads the
+    analysis and writes the trivial fission of rhs4center"""
+    import os
+    import shutil
+    import subprocess
+
+    if not shutil.which("gcc"):
+        pytest.skip("no C compiler")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    lib = os.path.join(root, "paper_conf_ipps_rawatvsrps19_b200", "lib")
+    exe = str(tmp_path / "c_api_host")
+    subprocess.check_call(["gcc", "-std=c99", "-Wall", "-Werror", "-I" + os.path.join(root, "include"),
+                           os.path.join(root, "examples", "c_api_host.c"), "-L" + lib, "-lsdag",
+                           "-Wl,-rpath," + lib, "-o", exe])
+    out = subprocess.run([exe, os.path.join(root, "paper_conf_ipps_rawatvsrps19_b200", "specs", "rhs4center.sdag")],
+                         capture_output=True, text=True, timeout=120)
+    assert out.returncode == 0, out.stderr
+    assert "dag jacobi7" in out.stdout and "radius 1 1 1 flops/pt 10" in out.stdout
+    assert "array B role 1" in out.stdout and "array A role 0" in out.stdout
+    assert "bad spec -> status 2 (PARSE)" in out.stdout
+    assert "trivial fission: 3 stencils" in out.stdout
