@@ -1,8 +1,9 @@
 """The C-ABI library loads without a GPU and exports every entry point that
-import pytest
 include/sdag.h declares (no compute calls)."""
 import os
 import re
+
+import pytest
 import subprocess
 
 import paper_conf_ipps_rawatvsrps19_b200 as sdag
