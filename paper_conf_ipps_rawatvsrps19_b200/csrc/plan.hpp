@@ -60,6 +60,14 @@ struct Plan {
     std::map<std::tuple<const void *, int64_t, int64_t, int64_t, int, int>, CUtensorMap> tmaps;
     std::vector<void *> ws;  // sdag_apply_host workspace (device buffers)
     std::vector<size_t> ws_bytes;
+    struct IterGraph {  // apply_iterated replays (CUDA graphs): key = buffers, T, scalars
+        std::string key;
+        cudaGraphExec_t exec = nullptr;
+        int launches = 0;
+    };
+    std::vector<IterGraph> graphs;  // guarded by graph_mu (not mu: capture enqueues launches, which take mu)
+    std::mutex graph_mu;
+    cudaStream_t cap_stream = nullptr;  // graph capture stream
     std::mutex host_mu;              // sdag_apply_host calls on one plan are serialised (shared workspace)
     cudaStream_t hs_up = nullptr;    // sdag_apply_host copy streams (H2D, D2H), created on first use
     cudaStream_t hs_down = nullptr;

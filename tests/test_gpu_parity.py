@@ -552,3 +552,35 @@ def test_temporal_fusion_exact_closed_form():
     assert sdag.launch_count() - n0 == 2  # two fused launches
     G = b0.cpu().numpy()
     assert np.array_equal(G, oracle.smooth27_iter(p, [-128.0, 14.0, 3.0, 1.0], 1 / 32, T))
+
+
+@pytest.mark.parametrize("name", ["jacobi7", "smooth27"])
+def test_iterated_cuda_graph_replay_is_bitwise(name, monkeypatch):
+    """launch-bound iterations are replayed as a CUDA graph (2nd call captures,
+    later calls replay): every call bitwise equal to plain launches, and the
+    launch counter still counts the sweeps' kernels"""
+    dims, T = (64, 64, 64), 12
+    case = make_case(name, (20, 21, 22))  # scalars only
+    s = case["s"]
+    A = synth.uniform(dims, -1.0, 1.0, "graph", name)
+    plan = sdag.Plan(sdag.spec_text(name), dims)
+    monkeypatch.setenv("SDAG_GRAPHS", "0")
+    r0 = torch.from_numpy(A).cuda()
+    r1 = r0.clone()
+    plan.apply_iterated(r0, r1, T, scalars=s)
+    torch.cuda.synchronize()
+    ref = r0.cpu().numpy()
+    n_plain = None
+    monkeypatch.setenv("SDAG_GRAPHS", "1")
+    b0 = torch.from_numpy(A).cuda()
+    b1 = b0.clone()
+    for call in range(4):  # plain, capture + replay, replay, replay
+        b0.copy_(torch.from_numpy(A))
+        b1.copy_(b0)
+        n0 = sdag.launch_count()
+        plan.apply_iterated(b0, b1, T, scalars=s)
+        torch.cuda.synchronize()
+        n = sdag.launch_count() - n0
+        n_plain = n if n_plain is None else n_plain
+        assert n == n_plain > 0, (call, n, n_plain)
+        assert np.array_equal(b0.cpu().numpy(), ref), call
