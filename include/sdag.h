@@ -190,7 +190,11 @@ void sdag_program_destroy(sdag_program prog);
  * with exactly one 3D input and one 3D output (and no 1D arrays):
  * sweep t reads buf[t&1] and writes the interior of buf[(t+1)&1].  Both
  * buffers must hold identical boundary rings on entry (fixed Dirichlet
- * ring).  Result in buf[T&1].
+ * ring).  Result in buf[T&1].  Sweeps may be fused per launch (temporal
+ * fusion, deep-tuning DP).  Launch-bound cases (<= 4 Mi interior points,
+ * T >= 4) are recorded as a CUDA graph on the second call with the same
+ * buffers, T and scalars and replayed afterwards (SDAG_GRAPHS=0 disables);
+ * the plan then holds the graph until it is destroyed.
  */
 sdag_status sdag_apply_iterated(sdag_plan plan, double *buf0, double *buf1, int32_t T, const double *scalars,
                                 int32_t nscalars, sdag_stream stream);
