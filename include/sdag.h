@@ -271,6 +271,9 @@ sdag_status sdag_dist_create(const char *spec, const int64_t global_dims[3], con
                              int32_t rank, int32_t nranks, void *nccl_comm, sdag_dist *out);
 /* local_dims = {nz_alloc, ny, nx}; global_z_of_local0 = global plane index of local plane 0 */
 sdag_status sdag_dist_layout(sdag_dist d, int64_t local_dims[3], int64_t *global_z_of_local0);
+/* The same, under the name of the SURVEY 8(b) boundary sketch: alloc_dims =
+ * {nz_owned + 2H, ny, nx}, *global_z0 = global plane of local plane 0. */
+sdag_status sdag_dist_alloc_dims(sdag_dist d, int64_t alloc_dims[3], int64_t *global_z0);
 sdag_plan sdag_dist_local_plan(sdag_dist d);
 
 /* One sweep of a slab: exchange the R_z boundary planes of every z-staged

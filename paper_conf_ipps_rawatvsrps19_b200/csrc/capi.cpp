@@ -296,6 +296,10 @@ sdag_status sdag_dist_layout(sdag_dist d, int64_t local_dims[3], int64_t *gz0) {
     });
 }
 
+sdag_status sdag_dist_alloc_dims(sdag_dist d, int64_t alloc_dims[3], int64_t *global_z0) {
+    return sdag_dist_layout(d, alloc_dims, global_z0);
+}
+
 sdag_plan sdag_dist_local_plan(sdag_dist d) {
     auto *D = reinterpret_cast<sdag::Dist *>(d);
     return D ? reinterpret_cast<sdag_plan>(&D->handle) : nullptr;
