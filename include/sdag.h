@@ -293,6 +293,14 @@ sdag_status sdag_dist_apply(sdag_dist d, double *const *arrays3d, int32_t n3d, c
 sdag_status sdag_dist_apply_iterated(sdag_dist d, double *buf0, double *buf1, int32_t T, const double *scalars,
                                      int32_t nscalars, sdag_stream compute, sdag_stream comm);
 void sdag_dist_destroy(sdag_dist d);
+/* One sweep of this rank's slab end to end with HOST buffers (local layout of
+ * sdag_dist_layout, ghost planes included: the host holds them, so no
+ * exchange is needed): pipelined H2D / sweep / D2H as sdag_apply_host; only
+ * the slab's planes of the global interior are computed and copied back (the
+ * rest of every output is not written).  Synchronous on `stream`. */
+sdag_status sdag_dist_apply_host(sdag_dist d, double *const *host3d, int32_t n3d, const double *const *host1d,
+                                 int32_t n1d, const double *scalars, int32_t nscalars, sdag_stream stream,
+                                 int64_t *h2d_bytes, int64_t *d2h_bytes);
 
 /* Loopback exchanger (all slabs in one process on one device; halos moved
  * with cudaMemcpyAsync): same index bookkeeping as the NCCL path, for

@@ -413,6 +413,21 @@ class Dist:
                                                             _stream_handle(stream)))
 
 
+    def apply_host(self, host3d, host1d=(), scalars=(), stream=None):
+        """One sweep of this slab end to end with host numpy buffers of the local
+        layout (ghost planes included): (h2d_bytes, d2h_bytes)"""
+        import numpy as np
+        for a in list(host3d) + list(host1d):
+            if not (isinstance(a, np.ndarray) and a.dtype == np.float64 and a.flags.c_contiguous):
+                raise TypeError("apply_host needs contiguous float64 numpy arrays")
+        p3 = [a.ctypes.data for a in host3d]
+        p1 = [a.ctypes.data for a in host1d]
+        s, ns = _scal(scalars)
+        up, down = ctypes.c_int64(), ctypes.c_int64()
+        _check(self._L.sdag_dist_apply_host(self._h, _arr(p3), len(p3), _arr(p1), len(p1), s, ns,
+                                            _stream_handle(stream), ctypes.byref(up), ctypes.byref(down)))
+        return up.value, down.value
+
     # ---- peer-memory halo path (NVLink P2P stores from the sweep kernels) ----
     def p2p_alloc(self):
         """(buf0, buf1): the library-owned slab buffers of sdag_dist_p2p_alloc as

@@ -332,6 +332,14 @@ sdag_status sdag_dist_apply_iterated_loopback(sdag_dist *dists, int32_t nranks, 
 
 void sdag_dist_destroy(sdag_dist d) { delete reinterpret_cast<sdag::Dist *>(d); }
 
+sdag_status sdag_dist_apply_host(sdag_dist d, double *const *h3, int32_t n3, const double *const *h1, int32_t n1,
+                                 const double *s, int32_t ns, sdag_stream stream, int64_t *h2d, int64_t *d2h) {
+    return guard([&] {
+        sdag::dist_apply_host(reinterpret_cast<sdag::Dist *>(d), h3, n3, h1, n1, s, ns,
+                              reinterpret_cast<cudaStream_t>(stream), h2d, d2h);
+    });
+}
+
 sdag_status sdag_spec_fission(const char *spec, int32_t kind, char *buf, int64_t cap, int64_t *len) {
     return guard([&] {
         if (!spec || !len) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null argument");

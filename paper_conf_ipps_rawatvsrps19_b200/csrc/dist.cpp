@@ -473,6 +473,14 @@ void p2p_map_peer(Dist *d, int side, void *base) {
 
 }  // namespace
 
+void dist_apply_host(Dist *d, double *const *h3, int n3, const double *const *h1, int n1, const double *s, int ns,
+                     cudaStream_t stream, int64_t *h2d, int64_t *d2h) {
+    if (!d) throw Error(SDAG_ERR_INVALID_ARG, "null dist");
+    if (d->local->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
+    const int64_t kr[2] = {d->slab.k_lo, d->slab.k_hi};
+    apply_host(d->local, h3, n3, h1, n1, s, ns, stream, h2d, d2h, kr);
+}
+
 void dist_p2p_alloc(Dist *d, double **buf0, double **buf1) {
     if (!d) throw Error(SDAG_ERR_INVALID_ARG, "null dist");
     if (d->local->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");

@@ -67,6 +67,12 @@ void dist_apply_iterated_loopback(Dist **d, int n, double *const *b0, double *co
 // peer-memory halo path (SURVEY 8(e) B200-native alternative): the launches
 // that compute a slab's boundary planes also store them into the neighbours'
 // ghost planes (NVLink P2P), ordered by per-neighbour flag words; no NCCL.
+// one sweep end to end with host buffers: the rank's host slab (local layout,
+// ghost planes included -- the host holds them) is pipelined H2D / sweep / D2H
+// like sdag_apply_host; only the rank's planes of the global interior are
+// computed and returned; no exchange is needed
+void dist_apply_host(Dist *d, double *const *h3, int n3, const double *const *h1, int n1, const double *s, int ns,
+                     cudaStream_t stream, int64_t *h2d, int64_t *d2h);
 void dist_p2p_alloc(Dist *d, double **buf0, double **buf1);
 void dist_p2p_handle(Dist *d, uint8_t handle[64]);
 void dist_p2p_attach(Dist *d, int side, const uint8_t handle[64]);

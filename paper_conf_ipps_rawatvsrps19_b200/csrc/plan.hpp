@@ -136,7 +136,8 @@ void plan_validate(Plan *p, double *const *a3, int n3, const double *const *a1, 
 std::vector<int> fusion_schedule(const double *f, int maxdeg, int T);
 void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int ns, cudaStream_t stream);
 void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int n1, const double *s, int ns,
-                cudaStream_t stream, int64_t *h2d, int64_t *d2h);
+                cudaStream_t stream, int64_t *h2d, int64_t *d2h,
+                const int64_t *krange = nullptr);
 void check_cuda(cudaError_t e, const char *what);
 // jit.cu (NEXT-4)
 std::string jit_body_source(const Plan &p, const std::string &sname, int rzr);

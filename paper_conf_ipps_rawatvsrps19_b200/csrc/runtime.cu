@@ -516,7 +516,7 @@ void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int
 // crosses the link once.  Outputs come back as the interior box only, so the
 // host ring is untouched.  Synchronous: returns after the last D2H.
 void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int n1, const double *s, int ns,
-                cudaStream_t stream, int64_t *h2d, int64_t *d2h) {
+                cudaStream_t stream, int64_t *h2d, int64_t *d2h, const int64_t *krange) {
     const int64_t nz = p->dims[0], ny = p->dims[1], nx = p->dims[2];
     const int64_t elems = nz * ny * nx, plane = ny * nx;
     if (n3 != p->n3() || n1 != p->n1() || ns != p->ns()) throw Error(SDAG_ERR_INVALID_ARG, "argument counts");
@@ -545,7 +545,10 @@ void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int
         }
     }
     const int64_t R = p->an.radius[0];
-    const int64_t zlo = p->lo[0], zhi = p->hi[0];
+    // output planes [zlo, zhi): the interior, or a sub-range (a z-slab's planes
+    // of the global interior, dist_apply_host)
+    const int64_t zlo = krange ? std::max<int64_t>(p->lo[0], krange[0]) : p->lo[0];
+    const int64_t zhi = krange ? std::min<int64_t>(p->hi[0], krange[1]) : p->hi[0];
     // chunks of >= 10 planes (and >= 2R_z so the halo share stays small), at
     // most 64: the pipeline fill (first upload) and drain (last download) are
     // one chunk each; measured on B200 at 512^3 (tools/e2e_probe.py): 16 chunks
