@@ -59,6 +59,8 @@ KernelDesc make_star_desc(const char *dag, int prio) {
                   TY, UY, PF, MINB > 1 ? (MINB == 2 ? "_mb2" : "_mb3") : "", unr);
     d.variant = buf;
     d.fn = reinterpret_cast<const void *>(&dev::sdag_star<B, TX, TY, UY, PF, TMA, QMODE, MINB, UNR>);
+    if constexpr (QMODE == 0)  // the dist p2p path's fused-store twin
+        d.fn_mirror = reinterpret_cast<const void *>(&dev::sdag_star<B, TX, TY, UY, PF, TMA, QMODE, MINB, UNR, true>);
     d.threads = G::THREADS;
     d.smem = G::SMEM;
     d.tx = TX;

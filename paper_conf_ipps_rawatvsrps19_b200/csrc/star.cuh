@@ -102,7 +102,8 @@ struct StarGeo {
     static_assert(PX <= 256 && PY <= 256, "TMA box");
 };
 
-template <class B, int TX, int TY, int UY, int PF, bool USE_TMA, int QMODE = 0, int MINB = 1, int UNR = 1>
+template <class B, int TX, int TY, int UY, int PF, bool USE_TMA, int QMODE = 0, int MINB = 1, int UNR = 1,
+          bool MIR = false>
 __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
     sdag_star(const __grid_constant__ SweepArgs a) {
     using G = StarGeo<B, TX, TY, UY, PF>;
@@ -367,15 +368,19 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
             release(k);  // last use of plane k (as centre)
             // interior-only streaming stores (16-B vector stores when both points are inside)
             double *o = a.out[0] + ((zbase + k) * a.ny + (y0 + cy)) * a.nx + gi;
+            const bool mp = MIR && mirror_plane(a, k);  // dist p2p: also into a neighbour's ghosts
 #pragma unroll
             for (int py = 0; py < UY; py++) {
                 // QMODE 3 (code differencing): arithmetic kept alive, stores (almost) never issued
                 if (py < nrows && (QMODE != 3 || acc[py][0] == 12345.678)) {
                     if (vec) {
                         __stcs(reinterpret_cast<double2 *>(o), make_double2(acc[py][0], acc[py][1]));
+                        if constexpr (MIR) if (mp) mirror2(a, k, o, acc[py][0], acc[py][1]);
                     } else {
                         if (ok0) __stcs(o, acc[py][0]);
                         if (ok1) __stcs(o + 1, acc[py][1]);
+                        if (MIR && mp && ok0) mirror1(a, k, o, acc[py][0]);
+                        if (MIR && mp && ok1) mirror1(a, k, o + 1, acc[py][1]);
                     }
                 }
                 o += a.nx;
