@@ -171,3 +171,18 @@ def test_gloo_slab_iteration_equals_global_oracle(P, tt, T):
     for _, z0, res in parts:
         got[z0:z0 + res.shape[0]] = res
     assert np.array_equal(got, ref)
+
+
+def test_p2p_entry_points_fail_cleanly_without_a_device():
+    """sdag_dist_p2p_* on a host-only slab: status codes, no crash (the peer
+    path itself is tests/test_gpu_p2p.py)"""
+    import paper_conf_ipps_rawatvsrps19_b200 as sdag
+    d = sdag.Dist(sdag.spec_text("smooth27"), (30, 20, 22), 0, 2, device=-2)
+    for call, code in ((lambda: d.p2p_alloc(), "DEVICE"), (lambda: d.p2p_handle(), "INVALID_ARG"),
+                       (lambda: d.p2p_attach(1, b"\0" * 64), "INVALID_ARG"),
+                       (lambda: d.p2p_apply_iterated(2, [0.0] * 5, stream=0), "INVALID_ARG")):
+        with pytest.raises(sdag.SdagError) as e:
+            call()
+        assert e.value.code == code
+    with pytest.raises(ValueError):
+        d.p2p_attach(1, b"short")
