@@ -447,10 +447,18 @@ def main():
     else:
         comm = None
         if not p2p:
-            uid = [sdag.nccl_unique_id() if rank == 0 else None]
+            uid = [None]
+            if rank == 0:
+                try:
+                    uid = [sdag.nccl_unique_id()]
+                except sdag.SdagError as e:  # no usable NCCL: the peer-memory halo needs none
+                    print(f"bench: NCCL halo unavailable ({e}); using the p2p halo", file=sys.stderr)
             if dist:
                 dist.broadcast_object_list(uid, src=0)
-            comm = sdag.nccl_comm_create(uid[0], world, rank, local)
+            if uid[0] is None:
+                p2p = True
+            else:
+                comm = sdag.nccl_comm_create(uid[0], world, rank, local)
         dd = sdag.Dist(spec, gdims, rank, world, comm=comm, tune=args.tune, variant=args.variant)
         (nza, ny, nx), g0 = dd.layout()
         part = sdag.slab_partition(gdims[0], 4, world, rank)
