@@ -187,7 +187,8 @@ struct Compiled {
     std::string log;
 };
 
-Compiled nvrtc_build(const std::string &src, const std::vector<std::string> &names, int maxrreg = 0) {
+Compiled nvrtc_build(const std::string &src, const std::vector<std::string> &names, int maxrreg = 0,
+                      bool strict = false) {
     const Nvrtc &N = nvrtc();
     nvrtcProgram prog;
     auto ck = [&](nvrtcResult r, const char *what) {
@@ -197,8 +198,9 @@ Compiled nvrtc_build(const std::string &src, const std::vector<std::string> &nam
     Compiled c;
     try {
         for (const auto &n : names) ck(N.add_name(prog, n.c_str()), "nvrtcAddNameExpression");
-        std::vector<const char *> opts = {"-arch=sm_100a", "-std=c++17", "-default-device", "--fmad=true",
-                                          "-lineinfo", "--extra-device-vectorization"};
+        std::vector<const char *> opts = {"-arch=sm_100a", "-std=c++17", "-default-device",
+                                          strict ? "--fmad=false" : "--fmad=true", "-lineinfo",
+                                          "--extra-device-vectorization"};
         const std::string rr = "--maxrregcount=" + std::to_string(maxrreg);
         if (maxrreg > 0) opts.push_back(rr.c_str());  // occupancy t: register rationing
         const nvrtcResult rc = N.compile(prog, int(opts.size()), opts.data());
@@ -385,8 +387,8 @@ void jit_build_candidates(Plan *p) {
         std::snprintf(buf, sizeof buf, "sdag::dev::sdag_sweep<sdag::dev::%s, %d, %d, %d, %d, %d, %s>", body, c.g.tx,
                       c.g.ty, c.g.ux, c.g.uy, c.g.pf, c.tma ? "true" : "false");
         names.push_back(buf);
-        std::snprintf(buf, sizeof buf, "jit_%s_%dx%d_u%dx%d_pf%d%s", c.tma ? "tma" : "lsu", c.g.tx, c.g.ty, c.g.ux,
-                      c.g.uy, c.g.pf, (c.rzr == RZ) ? "" : "_r0");
+        std::snprintf(buf, sizeof buf, "jit_%s_%dx%d_u%dx%d_pf%d%s%s", c.tma ? "tma" : "lsu", c.g.tx, c.g.ty, c.g.ux,
+                      c.g.uy, c.g.pf, (c.rzr == RZ) ? "" : "_r0", p->jit_strict ? "_strict" : "");
         c.name = buf;
     }
     for (CandQ &c : cq) {
@@ -394,8 +396,8 @@ void jit_build_candidates(Plan *p) {
         std::snprintf(buf, sizeof buf, "sdag::dev::sdag_sweepq<sdag::dev::JitBodyQ, %d, %d, %d, %d, %d, %s>", c.g.tx,
                       c.g.ty, c.g.ux, c.g.uy, c.g.pf, c.tma ? "true" : "false");
         names.push_back(buf);
-        std::snprintf(buf, sizeof buf, "jitq_%s_%dx%d_u%dx%d_pf%d", c.tma ? "tma" : "lsu", c.g.tx, c.g.ty, c.g.ux,
-                      c.g.uy, c.g.pf);
+        std::snprintf(buf, sizeof buf, "jitq_%s_%dx%d_u%dx%d_pf%d%s", c.tma ? "tma" : "lsu", c.g.tx, c.g.ty, c.g.ux,
+                      c.g.uy, c.g.pf, p->jit_strict ? "_strict" : "");
         c.name = buf;
     }
     const std::string key = src.str();
@@ -403,9 +405,10 @@ void jit_build_candidates(Plan *p) {
     std::lock_guard<std::mutex> lk(g_jit_mu);
     // compile (cached by source and register cap) and load on the plan's device
     auto build = [&](int cap) {
-        const std::string ck = cap ? key + "// --maxrregcount=" + std::to_string(cap) + "\n" : key;
+        const std::string ck = (cap ? key + "// --maxrregcount=" + std::to_string(cap) + "\n" : key) +
+                               (p->jit_strict ? "// --fmad=false\n" : "");
         auto it = g_compiled.find(ck);
-        if (it == g_compiled.end()) it = g_compiled.emplace(ck, nvrtc_build(key, names, cap)).first;
+        if (it == g_compiled.end()) it = g_compiled.emplace(ck, nvrtc_build(key, names, cap, p->jit_strict)).first;
         const Compiled &cc = it->second;
         std::vector<CUfunction> fns(names.size(), nullptr);
         if (p->host_only) return fns;

@@ -735,6 +735,10 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
     // compiled with NVRTC into the generic skeleton (jit.cu); host-only plans of
     // unregistered DAGs stay analysis-only unless "jit" is forced
     const bool forced_jit = p->force_variant.rfind("jit", 0) == 0;
+    // "jit_strict": program-order bodies compiled with --fmad=false -- the same
+    // IEEE operations as the oracle (R12), so results are bitwise the oracle's
+    p->jit_strict = forced_jit && p->force_variant.size() >= 7 &&
+                    p->force_variant.compare(p->force_variant.size() - 7, 7, "_strict") == 0;
     const bool use_jit = forced_jit || (!p->reg && !p->host_only);
     if (use_jit) {
         p->reg = nullptr;
@@ -758,7 +762,7 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
         jit_build_candidates(p.get());
         for (auto &k : p->jit_descs)
             if (!k->tma || p->dims[2] % 2 == 0) p->cands.push_back(k.get());
-        if (p->force_variant == "jit") p->force_variant.clear();
+        if (p->force_variant == "jit" || p->force_variant == "jit_strict") p->force_variant.clear();
     }
     for (const KernelDesc &k : kernel_table()) {
         if (use_jit) break;
