@@ -122,7 +122,7 @@ def test_batched_jacobi7():
     dims, batch = (16, 18, 20), 6
     ins, sc = synth.jacobi7_inputs(dims, cfg="batched", batch=batch)
     A = ins["A"]
-    plan = sdag.Plan(sdag.spec_text("jacobi7"), dims, batch=batch)
+    plan = sdag.Plan(sdag.spec_text("jacobi7"), dims, batch=batch, tune=tune)
     dA = torch.from_numpy(A).cuda()
     dB = torch.full(A.shape, float("nan"), dtype=torch.float64, device="cuda")
     plan.apply_batched(batch, [dB, dA], scalars=[sc["h2inv"], sc["a"], sc["b"]])
@@ -354,13 +354,14 @@ def _sample_points(dims, R, n, seed):
     return np.concatenate([pts, corners])
 
 
-def test_full_size_hypterm_sampled():
+@pytest.mark.parametrize("tune", [False, True])  # bench.py times the tune=1 plan of --config lines
+def test_full_size_hypterm_sampled(tune):
     """BASELINE config 3 (320^3) in bench.py's launch configuration, sampled."""
     dims = (320, 320, 320)
     case_ins, sc = synth.hypterm_inputs(dims)
     arrs = [case_ins[k] for k in ("cons_1", "cons_2", "cons_3", "cons_4", "q_1", "q_2", "q_3", "q_4")]
     s = [sc[k] for k in ("dxinv0", "dxinv1", "dxinv2", "ALP", "BET", "GAM", "DEL")]
-    plan = sdag.Plan(sdag.spec_text("hypterm"), dims)
+    plan = sdag.Plan(sdag.spec_text("hypterm"), dims, tune=tune)
     dev = [torch.from_numpy(a).cuda() for a in arrs]
     outs = [torch.full(dims, float("nan"), dtype=torch.float64, device="cuda") for _ in range(5)]
     plan.apply(outs + dev, scalars=s)
@@ -374,7 +375,8 @@ def test_full_size_hypterm_sampled():
     assert torch.isnan(outs[0][3, 100, 100]) and torch.isnan(outs[4][100, 100, 316])
 
 
-def test_full_size_rhs4_sampled():
+@pytest.mark.parametrize("tune", [False, True])  # bench.py times the tune=1 plan of --config lines
+def test_full_size_rhs4_sampled(tune):
     """BASELINE config 4 (320^3, uacc inout, a1 = 1), sampled."""
     dims = (320, 320, 320)
     ins, sc = synth.rhs4_inputs(dims)
@@ -382,7 +384,7 @@ def test_full_size_rhs4_sampled():
     ua = [ins["uacc0"], ins["uacc1"], ins["uacc2"]]
     a1d = [ins["strx"], ins["stry"], ins["strz"]]
     s = [sc[k] for k in ("tf", "i6", "i144", "cof", "a1")]
-    plan = sdag.Plan(sdag.spec_text("rhs4center"), dims)
+    plan = sdag.Plan(sdag.spec_text("rhs4center"), dims, tune=tune)
     d_ua = [torch.from_numpy(x.copy()).cuda() for x in ua]
     d_in = [torch.from_numpy(x).cuda() for x in (*u, ins["mu"], ins["la"])]
     plan.apply(d_ua + d_in, [torch.from_numpy(x).cuda() for x in a1d], s)
@@ -397,12 +399,13 @@ def test_full_size_rhs4_sampled():
     assert d_ua[0][0, 5, 5].item() == ua[0][0, 5, 5]  # ring untouched
 
 
-def test_full_size_jacobi7_batched_sampled():
+@pytest.mark.parametrize("tune", [False, True])  # bench.py times the tune=1 plan of --config lines
+def test_full_size_jacobi7_batched_sampled(tune):
     """BASELINE config 1b: 128 independent 64^3 problems in one launch."""
     dims, batch = (64, 64, 64), 128
     ins, sc = synth.jacobi7_inputs(dims, cfg="cfg1", batch=batch)
     A = ins["A"]
-    plan = sdag.Plan(sdag.spec_text("jacobi7"), dims, batch=batch)
+    plan = sdag.Plan(sdag.spec_text("jacobi7"), dims, batch=batch, tune=tune)
     dA = torch.from_numpy(A).cuda()
     dB = torch.full(A.shape, float("nan"), dtype=torch.float64, device="cuda")
     plan.apply_batched(batch, [dB, dA], scalars=[sc["h2inv"], sc["a"], sc["b"]])
@@ -416,7 +419,8 @@ def test_full_size_jacobi7_batched_sampled():
         assert np.isnan(G[b][0, 10, 10]) and np.isnan(G[b][10, 63, 10])
 
 
-def test_full_size_smooth27_iterated_sampled():
+@pytest.mark.parametrize("tune", [False, True])  # bench.py times the tune=1 plan of --config lines
+def test_full_size_smooth27_iterated_sampled(tune):
     """BASELINE config 5 on one GPU: 1024^3, T = 12 sweeps (the per-GPU slab of
     the weak-scaled run).  Input generated on the device by the same
     counter-based generator; the oracle evaluates sampled points from the
@@ -426,7 +430,7 @@ def test_full_size_smooth27_iterated_sampled():
     nu = 0.125
     b0 = synth.uniform_torch(dims, -1.0, 1.0, "cfg5", "A")
     b1 = b0.clone()
-    plan = sdag.Plan(sdag.spec_text("smooth27"), dims)
+    plan = sdag.Plan(sdag.spec_text("smooth27"), dims, tune=tune)
     plan.apply_iterated(b0, b1, T, scalars=[*w, nu])
     torch.cuda.synchronize()
     res = b0 if T % 2 == 0 else b1
