@@ -31,7 +31,11 @@ $(BUILD)/jit_embed.inc: $(SRC)/sweep.cuh tools/embed_text.py
 	@mkdir -p $(BUILD)
 	$(PY) tools/embed_text.py $@ kSweepSrc $(SRC)/sweep.cuh
 
-$(BUILD)/jit.o: $(BUILD)/jit_embed.inc
+$(BUILD)/jit_star_embed.inc: $(SRC)/star.cuh tools/embed_text.py
+	@mkdir -p $(BUILD)
+	$(PY) tools/embed_text.py $@ kStarSrc $(SRC)/star.cuh
+
+$(BUILD)/jit.o: $(BUILD)/jit_embed.inc $(BUILD)/jit_star_embed.inc
 
 $(BUILD)/%.o: $(SRC)/%.cpp $(HDRS)
 	@mkdir -p $(BUILD)

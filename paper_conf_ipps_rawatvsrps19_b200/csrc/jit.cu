@@ -40,7 +40,8 @@
 
 namespace sdag {
 
-#include "jit_embed.inc"  // kSweepSrc: the text of sweep.cuh
+#include "jit_embed.inc"       // kSweepSrc: the text of sweep.cuh
+#include "jit_star_embed.inc"  // kStarSrc: the text of star.cuh
 
 // ---------------------------------------------------------------------------
 // 1. code generation
@@ -118,6 +119,139 @@ std::string jit_body_source(const Plan &p, const std::string &sname, int rzr) {
     }
     for (int m = 0; m < nout; m++) o << "        o[" << m << "] = v" << m << ";\n";
     o << "    }\n};\n";
+    return o.str();
+}
+
+// ---------------------------------------------------------------------------
+// 1b. star form: a DAG that is LINEAR in its single input, with only on-axis
+// taps whose coefficients are mirror-symmetric (and equal for y and z), is
+// generated into the hand-written register-queue star kernel (star.cuh)
+// instead of the generic skeleton: B = K + c0 A + sum_r cx_r (A(+-r x)) +
+// cyz_r (A(+-r y) + A(+-r z)), coefficients any expressions of the scalars.
+// ---------------------------------------------------------------------------
+
+namespace {
+
+struct Lin {  // linear form over input taps: tap -> coefficient (C expression of scalars)
+    std::map<std::array<int, 3>, std::string> c;
+    std::string k;  // constant term ("" = none)
+    bool ok = true;
+};
+
+std::string cadd(const std::string &a, const std::string &b, char op) {
+    if (a.empty()) return op == '+' ? b : "(-" + b + ")";
+    if (b.empty()) return a;
+    return "(" + a + " " + op + " " + b + ")";
+}
+
+Lin lin_of(const Plan &p, int n, const std::vector<Lin> &temps) {
+    const Node &x = p.st.nodes[n];
+    Lin r;
+    auto is_const = [](const Lin &l) { return l.ok && l.c.empty(); };
+    switch (x.kind) {
+        case Node::Num: r.k = num_literal(x.value); return r;
+        case Node::Scalar: r.k = "a.s[" + std::to_string(x.ref) + "]"; return r;
+        case Node::Temp: return temps[x.ref];
+        case Node::Load3:
+            if (p.in_slot[x.ref] != 0 || p.n_staged != 1) r.ok = false;
+            else r.c[{x.off[0], x.off[1], x.off[2]}] = "(1.0)";
+            return r;
+        case Node::Load1: r.ok = false; return r;
+        case Node::Neg: {
+            Lin a = lin_of(p, x.a, temps);
+            for (auto &kv : a.c) kv.second = "(-" + kv.second + ")";
+            if (!a.k.empty()) a.k = "(-" + a.k + ")";
+            return a;
+        }
+        case Node::Add:
+        case Node::Sub: {
+            const char op = x.kind == Node::Add ? '+' : '-';
+            Lin a = lin_of(p, x.a, temps), b = lin_of(p, x.b, temps);
+            if (!a.ok || !b.ok) { r.ok = false; return r; }
+            r = a;
+            for (auto &kv : b.c) r.c[kv.first] = cadd(r.c.count(kv.first) ? r.c[kv.first] : "", kv.second, op);
+            if (!b.k.empty()) r.k = cadd(r.k, b.k, op);
+            return r;
+        }
+        case Node::Mul:
+        case Node::Div: {
+            Lin a = lin_of(p, x.a, temps), b = lin_of(p, x.b, temps);
+            if (!a.ok || !b.ok) { r.ok = false; return r; }
+            const char op = x.kind == Node::Mul ? '*' : '/';
+            if (is_const(b)) {  // (linear) op const
+                for (auto &kv : a.c) kv.second = "(" + kv.second + " " + op + " " + b.k + ")";
+                if (!a.k.empty()) a.k = "(" + a.k + " " + op + " " + b.k + ")";
+                return a;
+            }
+            if (op == '*' && is_const(a)) {
+                for (auto &kv : b.c) kv.second = "(" + a.k + " * " + kv.second + ")";
+                if (!b.k.empty()) b.k = "(" + a.k + " * " + b.k + ")";
+                return b;
+            }
+            r.ok = false;  // product or quotient of taps: not linear
+            return r;
+        }
+    }
+    r.ok = false;
+    return r;
+}
+
+}  // namespace
+
+// The star body for star.cuh, or "" when the DAG is not in star form.
+std::string jit_star_body(const Plan &p, int *R_out) {
+    if (p.an.n_in != 1 || p.n_staged != 1 || p.an.n_out != 1 || p.an.n_inout != 0 || p.n1() != 0) return "";
+    std::vector<Lin> temps(p.st.temps.size());
+    Lin out;
+    int writes = 0;
+    for (const Statement &st : p.st.stmts) {
+        Lin v = lin_of(p, st.expr, temps);
+        if (!v.ok) return "";
+        if (st.to_array) {
+            out = v;
+            writes++;
+        } else {
+            temps[st.target] = v;
+        }
+    }
+    if (writes != 1) return "";  // accumulating writes read the output: not this form
+    int R = 0;
+    for (auto &kv : out.c) {
+        const auto &t = kv.first;
+        const int nz = (t[0] != 0) + (t[1] != 0) + (t[2] != 0);
+        if (nz > 1) return "";  // off-axis tap
+        R = std::max({R, std::abs(t[0]), std::abs(t[1]), std::abs(t[2])});
+    }
+    if (R < 1 || R > 4) return "";
+    auto coef = [&](int dz, int dy, int dx) {
+        auto it = out.c.find({dz, dy, dx});
+        return it == out.c.end() ? std::string("(0.0)") : it->second;
+    };
+    std::ostringstream cx, cyz;
+    for (int r = 1; r <= R; r++) {
+        const std::string xp = coef(0, 0, r), xm = coef(0, 0, -r), yp = coef(0, r, 0), ym = coef(0, -r, 0),
+                          zp = coef(r, 0, 0), zm = coef(-r, 0, 0);
+        if (xp != xm || yp != ym || zp != zm || yp != zp) return "";  // not mirror / y-z symmetric
+        cx << "        case " << r << ": return " << xp << ";\n";
+        cyz << "        case " << r << ": return " << yp << ";\n";
+    }
+    *R_out = R;
+    std::ostringstream o;
+    o << "struct JitStar {\n"
+      << "    static constexpr int R = " << R << ", NIN = 1, NOUT = 1, NIO = 0, N1D = 0, RZ = " << R << ", RY = " << R
+      << ", RX = " << R << ", RZR = " << R << ";\n"
+      << "    __host__ __device__ static constexpr int axis1d(int) { return 2; }\n"
+      << "    __device__ __forceinline__ static double cx(const SweepArgs &a, int r) {\n"
+      << "        switch (r) {\n" << cx.str() << "        default: return 0.0;\n        }\n    }\n"
+      << "    __device__ __forceinline__ static double cyz(const SweepArgs &a, int r) {\n"
+      << "        switch (r) {\n" << cyz.str() << "        default: return 0.0;\n        }\n    }\n"
+      << "    __device__ __forceinline__ static void yz(double &acc, const SweepArgs &a, int r, double s) {\n"
+      << "        acc = fma(cyz(a, r), s, acc);\n    }\n"
+      << "    __device__ __forceinline__ static void x(double &acc, const SweepArgs &a, int r, double s) {\n"
+      << "        acc = fma(cx(a, r), s, acc);\n    }\n"
+      << "    __device__ __forceinline__ static double finish(double acc, const SweepArgs &a, double ctr) {\n"
+      << "        return fma(" << coef(0, 0, 0) << ", ctr, acc)" << (out.k.empty() ? "" : " + " + out.k) << ";\n"
+      << "    }\n};\n";
     return o.str();
 }
 
@@ -379,6 +513,34 @@ void jit_build_candidates(Plan *p) {
     if (need_r0 && RZ > 0) src << jit_body_source(*p, "JitBodyR0", 0);
     if (need_r0 && RZ == 0 && !need_full) src << jit_body_source(*p, "JitBody", 0);
     if (!cq.empty()) src << jit_body_source(*p, "JitBodyQ", rz_off);
+    // star form (linear, on-axis, mirror-symmetric): the hand-written star kernel
+    int Rstar = 0;
+    const std::string star_body = (p->st.pragma.block[0] > 0 || p->st.pragma.occupancy > 0 || p->jit_strict)
+                                      ? std::string()  // user guidance / strict order: the generic skeleton
+                                      : jit_star_body(*p, &Rstar);
+    struct CandS {
+        int tx, ty, uy, pf, unr;
+        std::string name;
+        int smem, threads;
+    };
+    std::vector<CandS> cst;
+    p->jit_star_src = star_body;
+    if (!star_body.empty()) {
+        src << "}  // namespace dev\n}  // namespace sdag\n" << kStarSrc << "\nnamespace sdag {\nnamespace dev {\n"
+            << star_body;
+        // the registered star geometries (lap25 / jacobi7 measured picks, DESIGN 6.3)
+        const int cfgs[2][5] = {{32, 32, 4, 3, 2}, {64, 16, 2, 3, 1}};
+        for (const auto &g : cfgs) {
+            const int ML = Rstar + (Rstar % 2), px = g[0] + 2 * ML, py = g[1] + 2 * Rstar;
+            const int plane_al = ((px * py * 8 + 127) / 128) * 128 / 8, ns = Rstar + 1 + g[3];
+            const int smem = ns * plane_al * 8 + 2 * ns * 8;
+            if (px > 256 || py > 256 || smem > 227 * 1024) continue;
+            char buf[96];
+            std::snprintf(buf, sizeof buf, "jitstar_tma_%dx%d_u2x%d_pf%d%s", g[0], g[1], g[2], g[3],
+                          g[4] > 1 ? "_z2" : "");
+            cst.push_back({g[0], g[1], g[2], g[3], g[4], buf, smem, (g[0] / 2) * (g[1] / g[2])});
+        }
+    }
     src << "}  // namespace dev\n}  // namespace sdag\n";
     std::vector<std::string> names;
     for (Cand &c : cs) {
@@ -399,6 +561,12 @@ void jit_build_candidates(Plan *p) {
         std::snprintf(buf, sizeof buf, "jitq_%s_%dx%d_u%dx%d_pf%d%s", c.tma ? "tma" : "lsu", c.g.tx, c.g.ty, c.g.ux,
                       c.g.uy, c.g.pf, p->jit_strict ? "_strict" : "");
         c.name = buf;
+    }
+    for (CandS &c : cst) {
+        char buf[200];
+        std::snprintf(buf, sizeof buf, "sdag::dev::sdag_star<sdag::dev::JitStar, %d, %d, %d, %d, true, 0, 1, %d>", c.tx,
+                      c.ty, c.uy, c.pf, c.unr);
+        names.push_back(buf);
     }
     const std::string key = src.str();
 
@@ -488,6 +656,31 @@ void jit_build_candidates(Plan *p) {
         d->rx = RX;
         d->rzr = rz_off;
         d->prio = -10 + int(q / 2) + (c.tma ? 0 : 100);  // preferred: 1.35x (lap25), 1.1x (27-pt) over the ring-only skeleton
+        p->jit_descs.push_back(std::move(d));
+    }
+
+    for (size_t q = 0; q < cst.size(); q++) {
+        const CandS &c = cst[q];
+        auto d = std::make_unique<KernelDesc>();
+        d->dag = "(jit)";
+        d->variant = c.name;
+        d->fn = nullptr;
+        d->cufn = fns[cs.size() + cq.size() + q];
+        d->threads = c.threads;
+        d->smem = c.smem;
+        d->tx = c.tx;
+        d->ty = c.ty;
+        d->ux = 2;
+        d->uy = c.uy;
+        d->pf = c.pf;
+        d->tma = true;
+        d->nin = 1;
+        d->nout = 1;
+        d->rz = Rstar;
+        d->ry = Rstar;
+        d->rx = Rstar + (Rstar % 2);  // TMA box margin (star.cuh ML)
+        d->rzr = Rstar;
+        d->prio = -20 + int(q);  // the register-queue star kernel first
         p->jit_descs.push_back(std::move(d));
     }
 

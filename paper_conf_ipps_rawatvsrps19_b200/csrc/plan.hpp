@@ -42,7 +42,8 @@ struct Plan {
     // ABI mapping (per 3D formal kind_index): staged-input slot / output slot / inout slot
     std::vector<int> in_slot, out_slot, io_slot;
     int jit_maxrreg = 0;
-    bool jit_strict = false;  // force_variant "jit_strict": generated kernels without FMA contraction
+    bool jit_strict = false;
+    std::string jit_star_src;  // generated star-kernel body when the DAG is in star form (jit.cu)  // force_variant "jit_strict": generated kernels without FMA contraction
     int zchunk_tuned = 0;   // z-chunk length chosen by tune=1 (0 = the occupancy model's)
     int tuned_timed = 0;    // candidates timed by the hierarchical tuner  // --maxrregcount of the generated kernels (occupancy t), 0 = none
     int n_staged = 0;  // inputs staged in shared memory: slots [0, n_staged); generated kernels

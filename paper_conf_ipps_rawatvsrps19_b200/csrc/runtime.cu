@@ -846,6 +846,9 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
               << " staged";
         }
     }
+    if (!p->jit_star_src.empty())
+        d << "\n  star form: linear, on-axis, mirror-symmetric -> the register-queue star kernel (star.cuh):\n"
+          << p->jit_star_src;
     if (!p->jit_descs.empty())
         d << "\n  jit body (NVRTC, sm_100a, into the sweep.cuh skeleton):\n" << jit_body_source(*p, "JitBody", p->an.radius[0]);
     p->describe_text = d.str();

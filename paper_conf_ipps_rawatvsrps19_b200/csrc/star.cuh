@@ -38,9 +38,21 @@
 // error gate (reading R13).
 #pragma once
 
+#ifdef __CUDACC_RTC__
+// NVRTC (jit.cu): sweep.cuh's text precedes this one; the one std facility used
+namespace std {
+template <class T, T v>
+struct integral_constant {
+    static constexpr T value = v;
+    using value_type = T;
+    constexpr operator T() const { return v; }
+};
+}  // namespace std
+#else
 #include <type_traits>
 
 #include "sweep.cuh"
+#endif
 
 namespace sdag {
 namespace dev {
