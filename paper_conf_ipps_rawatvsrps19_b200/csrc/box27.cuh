@@ -42,6 +42,10 @@ struct BoxGeo {
 };
 
 // FORM 0: the 27-point smoother (scalars w0..w3, nu).
+// FORM 2: any linear 27-point box stencil whose weights depend only on the tap
+//   class (centre, face, edge, corner): B = w0 A + w1 faces + w2 edges + w3
+//   corners, w0..w3 in s[0..3] (generated DAGs in box form, jit.cu; the
+//   weights are evaluated from the DAG's scalars at launch).
 // FORM 1: Listing 1's 7-point Jacobi (scalars h2inv, a, b) in the same
 //   retimed form: T_k = s1_k - 6 s0_k + s0_{k-1} is formed when plane k
 //   streams past and B[k] = a A[k] - (b h2inv)(T_k + s0_{k+1}) when plane k+1
@@ -164,11 +168,14 @@ __global__ void __launch_bounds__(BoxGeo<TX, TY, UY, PF>::THREADS)
                 const int c = ML + px;  // centre column in w
                 const double s0 = w[py + 1][c];
                 const double s1 = (w[py + 1][c - 1] + w[py + 1][c + 1]) + (w[py][c] + w[py + 2][c]);
-                if constexpr (FORM == 0) {
+                if constexpr (FORM == 0 || FORM == 2) {
                     const double s2 = (w[py][c - 1] + w[py][c + 1]) + (w[py + 2][c - 1] + w[py + 2][c + 1]);
                     const double cc = fma(w2, s2, fma(w1, s1, w0 * s0));
                     const double uu = fma(w3, s2, fma(w2, s1, w1 * s0));
-                    res[px] = fma(nu, Tprev[py][px] + uu, Aprev[py][px]);  // B[k] = A[k] + nu(u_{k-1} + c_k + u_{k+1})
+                    if constexpr (FORM == 0)
+                        res[px] = fma(nu, Tprev[py][px] + uu, Aprev[py][px]);  // B[k] = A[k] + nu(u_{k-1} + c_k + u_{k+1})
+                    else
+                        res[px] = Tprev[py][px] + uu;  // FORM 2: B[k] = u_{k-1} + c_k + u_{k+1}
                     Tprev[py][px] = Uprev[py][px] + cc;                   // u_{p-1} + c_p
                     Uprev[py][px] = uu;
                 } else {

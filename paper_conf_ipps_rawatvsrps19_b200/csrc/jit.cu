@@ -198,6 +198,108 @@ Lin lin_of(const Plan &p, int n, const std::vector<Lin> &temps) {
 
 }  // namespace
 
+// Box form: linear in the one input, taps within the 3x3x3 box, the
+// coefficient of a tap depending only on its class (centre / face / edge /
+// corner, by the number of nonzero offsets) -> the retimed, folded box27
+// kernel (FORM 2).  Weights w0..w3 (expressions of the scalars) are evaluated
+// on the host at each launch.  Returns false when the DAG is not in box form.
+bool jit_box_form(const Plan &p, std::vector<std::string> &w) {
+    if (p.an.n_in != 1 || p.n_staged != 1 || p.an.n_out != 1 || p.an.n_inout != 0 || p.n1() != 0) return false;
+    if (p.an.radius[0] != 1 || p.an.radius[1] != 1 || p.an.radius[2] != 1) return false;
+    std::vector<Lin> temps(p.st.temps.size());
+    Lin out;
+    int writes = 0;
+    for (const Statement &st : p.st.stmts) {
+        Lin v = lin_of(p, st.expr, temps);
+        if (!v.ok) return false;
+        if (st.to_array) {
+            out = v;
+            writes++;
+        } else {
+            temps[st.target] = v;
+        }
+    }
+    if (writes != 1 || !out.k.empty()) return false;
+    std::string cls[4];
+    bool seen[4] = {false, false, false, false};
+    for (int dz = -1; dz <= 1; dz++)
+        for (int dy = -1; dy <= 1; dy++)
+            for (int dx = -1; dx <= 1; dx++) {
+                const int c = (dz != 0) + (dy != 0) + (dx != 0);
+                auto it = out.c.find({dz, dy, dx});
+                const std::string v = it == out.c.end() ? "(0.0)" : it->second;
+                if (!seen[c]) {
+                    cls[c] = v;
+                    seen[c] = true;
+                } else if (cls[c] != v) {
+                    return false;
+                }
+            }
+    w.assign(cls, cls + 4);
+    return true;
+}
+
+namespace {
+struct CoefEval {  // recursive descent over the generated coefficient text
+    const char *q;
+    const double *s;
+    int ns;
+    void ws() {
+        while (*q == ' ') q++;
+    }
+    double factor() {
+        ws();
+        if (*q == '(') {
+            q++;
+            const double v = expr();
+            ws();
+            if (*q != ')') throw Error(SDAG_ERR_INVALID_ARG, "coefficient: ')' expected");
+            q++;
+            return v;
+        }
+        if (*q == '-') {
+            q++;
+            return -factor();
+        }
+        if (std::strncmp(q, "a.s[", 4) == 0) {
+            q += 4;
+            const int i = int(std::strtol(q, const_cast<char **>(&q), 10));
+            if (*q != ']' || i < 0 || i >= ns) throw Error(SDAG_ERR_INVALID_ARG, "coefficient: bad scalar index");
+            q++;
+            return s[i];
+        }
+        char *end = nullptr;
+        const double v = std::strtod(q, &end);
+        if (end == q) throw Error(SDAG_ERR_INVALID_ARG, "coefficient: number expected");
+        q = end;
+        return v;
+    }
+    double term() {
+        double v = factor();
+        for (;;) {
+            ws();
+            if (*q == '*') q++, v = v * factor();
+            else if (*q == '/') q++, v = v / factor();
+            else return v;
+        }
+    }
+    double expr() {
+        double v = term();
+        for (;;) {
+            ws();
+            if (*q == '+') q++, v = v + term();
+            else if (*q == '-') q++, v = v - term();
+            else return v;
+        }
+    }
+};
+}  // namespace
+
+double jit_eval_coef(const std::string &e, const double *s, int ns) {
+    CoefEval c{e.c_str(), s, ns};
+    return c.expr();
+}
+
 // The star body for star.cuh, or "" when the DAG is not in star form.
 std::string jit_star_body(const Plan &p, int *R_out) {
     if (p.an.n_in != 1 || p.n_staged != 1 || p.an.n_out != 1 || p.an.n_inout != 0 || p.n1() != 0) return "";
@@ -525,6 +627,9 @@ void jit_build_candidates(Plan *p) {
     };
     std::vector<CandS> cst;
     p->jit_star_src = star_body;
+    p->box_w.clear();
+    if (star_body.empty() && !(p->st.pragma.block[0] > 0 || p->st.pragma.occupancy > 0 || p->jit_strict))
+        jit_box_form(*p, p->box_w);
     if (!star_body.empty()) {
         src << "}  // namespace dev\n}  // namespace sdag\n" << kStarSrc << "\nnamespace sdag {\nnamespace dev {\n"
             << star_body;

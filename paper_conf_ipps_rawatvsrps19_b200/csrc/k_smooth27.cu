@@ -5,6 +5,11 @@
 namespace sdag {
 void add_kernels_smooth27(std::vector<KernelDesc> &v) {
     SDAG_BOX_PAIR(v, "smooth27", 128, 16, 4, 2, 0);
+    // FORM 2 (generated DAGs in box form, jit.cu): weights by tap class
+    // (preferred over every generated candidate of such a plan: negative priorities)
+    v.push_back(make_box27_desc<128, 16, 4, 2, true, 2>("(box27)", -40));
+    v.push_back(make_box27_desc<128, 16, 4, 2, false, 2>("(box27)", 60));
+    v.push_back(make_box27_desc<64, 32, 4, 3, true, 2>("(box27)", -39));
     SDAG_BOX_PAIR(v, "smooth27", 64, 32, 4, 3, 1);
     SDAG_BOX_PAIR(v, "smooth27", 64, 16, 4, 3, 2);
     SDAG_BOX_PAIR(v, "smooth27", 128, 16, 4, 3, 3);

@@ -86,8 +86,8 @@ KernelDesc make_box27_desc(const char *dag, int prio) {
     KernelDesc d;
     d.dag = dag;
     char buf[96];
-    std::snprintf(buf, sizeof buf, "%s_%s_%dx%d_u2x%d_pf%d", FORM ? "cross" : "box", TMA ? "tma" : "lsu", TX, TY, UY,
-                  PF);
+    std::snprintf(buf, sizeof buf, "%s_%s_%dx%d_u2x%d_pf%d", FORM == 1 ? "cross" : (FORM == 2 ? "jitbox" : "box"),
+                  TMA ? "tma" : "lsu", TX, TY, UY, PF);
     d.variant = buf;
     d.fn = reinterpret_cast<const void *>(&dev::sdag_box27<TX, TY, UY, PF, TMA, FORM>);
     d.fn_mirror = reinterpret_cast<const void *>(&dev::sdag_box27<TX, TY, UY, PF, TMA, FORM, true>);

@@ -43,7 +43,8 @@ struct Plan {
     std::vector<int> in_slot, out_slot, io_slot;
     int jit_maxrreg = 0;
     bool jit_strict = false;
-    std::string jit_star_src;  // generated star-kernel body when the DAG is in star form (jit.cu)  // force_variant "jit_strict": generated kernels without FMA contraction
+    std::string jit_star_src;  // generated star-kernel body when the DAG is in star form (jit.cu)
+    std::vector<std::string> box_w;  // box form: class weights w0..w3 as expressions of a.s[] (jit.cu)  // force_variant "jit_strict": generated kernels without FMA contraction
     int zchunk_tuned = 0;   // z-chunk length chosen by tune=1 (0 = the occupancy model's)
     int tuned_timed = 0;    // candidates timed by the hierarchical tuner  // --maxrregcount of the generated kernels (occupancy t), 0 = none
     int n_staged = 0;  // inputs staged in shared memory: slots [0, n_staged); generated kernels
@@ -144,6 +145,8 @@ void check_cuda(cudaError_t e, const char *what);
 // jit.cu (NEXT-4)
 std::string jit_body_source(const Plan &p, const std::string &sname, int rzr);
 void jit_build_candidates(Plan *p);
+// box form (jit.cu): evaluate a weight expression over the call's scalars
+double jit_eval_coef(const std::string &e, const double *s, int ns);
 void jit_launch(const KernelDesc &k, dim3 grid, void **args, cudaStream_t stream);
 int jit_occupancy(const KernelDesc &k);
 

@@ -256,6 +256,10 @@ void plan_launch(Plan *p, const KernelDesc &k, double *const *a3, const double *
     int ns = 0;
     for (int q = 0; q < p->ns(); q++) A.s[ns++] = s[q];
     for (double e : p->extra_scalars) A.s[ns++] = e;
+    if (k.dag == "(box27)") {  // box form: class weights from the DAG's scalars
+        if (p->box_w.size() != 4) throw Error(SDAG_ERR_INVALID_ARG, "box kernel on a plan not in box form");
+        for (int q = 0; q < 4; q++) A.s[q] = jit_eval_coef(p->box_w[q], s, p->ns());
+    }
     A.nx = dims[2];
     A.ny = dims[1];
     A.nz = dims[0];
@@ -762,6 +766,9 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
         jit_build_candidates(p.get());
         for (auto &k : p->jit_descs)
             if (!k->tma || p->dims[2] % 2 == 0) p->cands.push_back(k.get());
+        if (!p->box_w.empty())  // box form: the hand-written box kernel, FORM 2
+            for (const KernelDesc &k : kernel_table())
+                if (k.dag == "(box27)" && (!k.tma || p->dims[2] % 2 == 0)) p->cands.push_back(&k);
         if (p->force_variant == "jit" || p->force_variant == "jit_strict") p->force_variant.clear();
     }
     for (const KernelDesc &k : kernel_table()) {
@@ -846,6 +853,10 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
               << " staged";
         }
     }
+    if (!p->box_w.empty())
+        d << "\n  box form: linear, 3x3x3, weights by tap class -> the retimed/folded box kernel (box27.cuh FORM 2);"
+          << " w0..w3 = " << p->box_w[0] << ", " << p->box_w[1] << ", " << p->box_w[2] << ", " << p->box_w[3]
+          << " (evaluated at launch)";
     if (!p->jit_star_src.empty())
         d << "\n  star form: linear, on-axis, mirror-symmetric -> the register-queue star kernel (star.cuh):\n"
           << p->jit_star_src;
