@@ -122,7 +122,7 @@ def test_batched_jacobi7():
     dims, batch = (16, 18, 20), 6
     ins, sc = synth.jacobi7_inputs(dims, cfg="batched", batch=batch)
     A = ins["A"]
-    plan = sdag.Plan(sdag.spec_text("jacobi7"), dims, batch=batch, tune=tune)
+    plan = sdag.Plan(sdag.spec_text("jacobi7"), dims, batch=batch)
     dA = torch.from_numpy(A).cuda()
     dB = torch.full(A.shape, float("nan"), dtype=torch.float64, device="cuda")
     plan.apply_batched(batch, [dB, dA], scalars=[sc["h2inv"], sc["a"], sc["b"]])
