@@ -47,7 +47,8 @@ struct Fuse2Geo {
 // UX = 2 or 4 output columns per thread: the row window of a UX-wide patch is
 // UX+4 doubles read with (UX+4)/2 128-bit loads, so UX = 4 cuts the fold's
 // shared-memory reads per point from 1.5 to 1 LDS.128 per row.
-// FORM 0: the 27-point smoother (scalars w0..w3, nu);
+// FORM 0: the 27-point smoother (scalars w0..w3, nu); FORM 2: a generated
+//   box-form DAG, B = w0 A + w1 faces + w2 edges + w3 corners (box27.cuh);
 // FORM 1: Listing 1's 7-point Jacobi (scalars h2inv, a, b), the paper's
 //   7pt-smoother of Table I / Table II, in box27's retimed FORM 1:
 //   T_k = s1_k - 6 s0_k + s0_{k-1}, B[k] = a A[k] - (b h2inv)(T_k + s0_{k+1}).
@@ -148,7 +149,7 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
                 const int c = ML - W0 + px;  // the patch point's column in the window
                 const double s0 = w[py + 1][c];
                 const double s1 = (w[py + 1][c - 1] + w[py + 1][c + 1]) + (w[py][c] + w[py + 2][c]);
-                if constexpr (FORM == 0) {
+                if constexpr (FORM == 0 || FORM == 2) {
                     const double s2 = (w[py][c - 1] + w[py][c + 1]) + (w[py + 2][c - 1] + w[py + 2][c + 1]);
                     cc[py][px] = fma(w2, s2, fma(w1, s1, w0 * s0));
                     uu[py][px] = fma(w3, s2, fma(w2, s1, w1 * s0));
@@ -178,8 +179,8 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
             double v[UX];
 #pragma unroll
             for (int px = 0; px < UX; px++) {
-                if constexpr (FORM == 0) {
-                    v[px] = fma(nu, T1[py][px] + uu[py][px], A1[py][px]);
+                if constexpr (FORM == 0 || FORM == 2) {
+                    v[px] = FORM == 0 ? fma(nu, T1[py][px] + uu[py][px], A1[py][px]) : T1[py][px] + uu[py][px];
                     T1[py][px] = U1[py][px] + cc[py][px];
                     U1[py][px] = uu[py][px];
                 } else {
@@ -212,8 +213,8 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
             double res[UX];
 #pragma unroll
             for (int px = 0; px < UX; px++) {
-                if constexpr (FORM == 0) {
-                    res[px] = fma(nu, T2[py][px] + uu[py][px], A2[py][px]);
+                if constexpr (FORM == 0 || FORM == 2) {
+                    res[px] = FORM == 0 ? fma(nu, T2[py][px] + uu[py][px], A2[py][px]) : T2[py][px] + uu[py][px];
                     T2[py][px] = U2[py][px] + cc[py][px];
                     U2[py][px] = uu[py][px];
                 } else {

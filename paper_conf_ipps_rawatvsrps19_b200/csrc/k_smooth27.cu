@@ -10,6 +10,8 @@ void add_kernels_smooth27(std::vector<KernelDesc> &v) {
     v.push_back(make_box27_desc<128, 16, 4, 2, true, 2>("(box27)", -40));
     v.push_back(make_box27_desc<128, 16, 4, 2, false, 2>("(box27)", 60));
     v.push_back(make_box27_desc<64, 32, 4, 3, true, 2>("(box27)", -39));
+    v.push_back(make_fuse2_desc<64, 16, 2, 2, 2, 2, true, 2>("(box27)", -40));  // temporal fusion, FORM 2
+    v.back().fhint = 1.69;
     SDAG_BOX_PAIR(v, "smooth27", 64, 32, 4, 3, 1);
     SDAG_BOX_PAIR(v, "smooth27", 64, 16, 4, 3, 2);
     SDAG_BOX_PAIR(v, "smooth27", 128, 16, 4, 3, 3);

@@ -766,9 +766,14 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
         jit_build_candidates(p.get());
         for (auto &k : p->jit_descs)
             if (!k->tma || p->dims[2] % 2 == 0) p->cands.push_back(k.get());
-        if (!p->box_w.empty())  // box form: the hand-written box kernel, FORM 2
-            for (const KernelDesc &k : kernel_table())
-                if (k.dag == "(box27)" && (!k.tma || p->dims[2] % 2 == 0)) p->cands.push_back(&k);
+        if (!p->box_w.empty())  // box form: the hand-written box kernels, FORM 2 (single and fused sweeps)
+            for (const KernelDesc &k : kernel_table()) {
+                if (k.dag != "(box27)" || (k.tma && p->dims[2] % 2 != 0)) continue;
+                if (k.tsteps > 1)
+                    p->fused.push_back(&k);
+                else
+                    p->cands.push_back(&k);
+            }
         if (p->force_variant == "jit" || p->force_variant == "jit_strict") p->force_variant.clear();
     }
     for (const KernelDesc &k : kernel_table()) {
