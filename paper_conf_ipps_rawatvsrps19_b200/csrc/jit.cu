@@ -627,15 +627,15 @@ void jit_build_candidates(Plan *p) {
     };
     std::vector<CandS> cst;
     p->jit_star_src = star_body;
-    p->box_w.clear();
-    if (star_body.empty() && !(p->st.pragma.block[0] > 0 || p->st.pragma.occupancy > 0 || p->jit_strict))
-        jit_box_form(*p, p->box_w);
+    p->box_w.clear();  // (a radius-1 star is also in box form: box kernels + temporal fusion, star kernels too)
+    if (!(p->st.pragma.block[0] > 0 || p->st.pragma.occupancy > 0 || p->jit_strict)) jit_box_form(*p, p->box_w);
     if (!star_body.empty()) {
         src << "}  // namespace dev\n}  // namespace sdag\n" << kStarSrc << "\nnamespace sdag {\nnamespace dev {\n"
             << star_body;
         // the registered star geometries (lap25 / jacobi7 measured picks, DESIGN 6.3)
-        const int cfgs[2][5] = {{32, 32, 4, 3, 2}, {64, 16, 2, 3, 1}};
-        for (const auto &g : cfgs) {
+        // (radius <= 2: Jacobi's 64x16 first; wider radii: the Laplacian's 32x32)
+        const int big[2][5] = {{32, 32, 4, 3, 2}, {64, 16, 2, 3, 1}}, small[2][5] = {{64, 16, 2, 3, 1}, {32, 32, 4, 3, 2}};
+        for (const auto &g : (Rstar <= 2 ? small : big)) {
             const int ML = Rstar + (Rstar % 2), px = g[0] + 2 * ML, py = g[1] + 2 * Rstar;
             const int plane_al = ((px * py * 8 + 127) / 128) * 128 / 8, ns = Rstar + 1 + g[3];
             const int smem = ns * plane_al * 8 + 2 * ns * 8;
@@ -785,7 +785,7 @@ void jit_build_candidates(Plan *p) {
         d->ry = Rstar;
         d->rx = Rstar + (Rstar % 2);  // TMA box margin (star.cuh ML)
         d->rzr = Rstar;
-        d->prio = -20 + int(q);  // the register-queue star kernel first
+        d->prio = -50 + int(q);  // the register-queue star kernel first (before box kernels: radius-1 stars)
         p->jit_descs.push_back(std::move(d));
     }
 
