@@ -329,26 +329,36 @@ std::string jit_star_body(const Plan &p, int *R_out) {
         auto it = out.c.find({dz, dy, dx});
         return it == out.c.end() ? std::string("(0.0)") : it->second;
     };
-    std::ostringstream cx, cyz;
+    std::ostringstream cx, cyz, cz;
+    bool split = false;
     for (int r = 1; r <= R; r++) {
         const std::string xp = coef(0, 0, r), xm = coef(0, 0, -r), yp = coef(0, r, 0), ym = coef(0, -r, 0),
                           zp = coef(r, 0, 0), zm = coef(-r, 0, 0);
-        if (xp != xm || yp != ym || zp != zm || yp != zp) return "";  // not mirror / y-z symmetric
+        if (xp != xm || yp != ym || zp != zm) return "";  // not mirror-symmetric
+        if (yp != zp) split = true;                      // distinct y and z coefficients
         cx << "        case " << r << ": return " << xp << ";\n";
         cyz << "        case " << r << ": return " << yp << ";\n";
+        cz << "        case " << r << ": return " << zp << ";\n";
     }
     *R_out = R;
     std::ostringstream o;
     o << "struct JitStar {\n"
       << "    static constexpr int R = " << R << ", NIN = 1, NOUT = 1, NIO = 0, N1D = 0, RZ = " << R << ", RY = " << R
       << ", RX = " << R << ", RZR = " << R << ";\n"
+      << "    static constexpr bool SPLIT_YZ = " << (split ? "true" : "false") << ";\n"
       << "    __host__ __device__ static constexpr int axis1d(int) { return 2; }\n"
       << "    __device__ __forceinline__ static double cx(const SweepArgs &a, int r) {\n"
       << "        switch (r) {\n" << cx.str() << "        default: return 0.0;\n        }\n    }\n"
       << "    __device__ __forceinline__ static double cyz(const SweepArgs &a, int r) {\n"
       << "        switch (r) {\n" << cyz.str() << "        default: return 0.0;\n        }\n    }\n"
+      << "    __device__ __forceinline__ static double cz(const SweepArgs &a, int r) {\n"
+      << "        switch (r) {\n" << cz.str() << "        default: return 0.0;\n        }\n    }\n"
       << "    __device__ __forceinline__ static void yz(double &acc, const SweepArgs &a, int r, double s) {\n"
       << "        acc = fma(cyz(a, r), s, acc);\n    }\n"
+      << "    __device__ __forceinline__ static void y(double &acc, const SweepArgs &a, int r, double s) {\n"
+      << "        acc = fma(cyz(a, r), s, acc);\n    }\n"
+      << "    __device__ __forceinline__ static void z(double &acc, const SweepArgs &a, int r, double s) {\n"
+      << "        acc = fma(cz(a, r), s, acc);\n    }\n"
       << "    __device__ __forceinline__ static void x(double &acc, const SweepArgs &a, int r, double s) {\n"
       << "        acc = fma(cx(a, r), s, acc);\n    }\n"
       << "    __device__ __forceinline__ static double finish(double acc, const SweepArgs &a, double ctr) {\n"

@@ -60,6 +60,7 @@ namespace dev {
 // 25-point radius-4 Laplacian: B = c0*A + sum_r c_r*(6 taps at distance r)
 struct Lap25Star {
     static constexpr int R = 4, NIN = 1, NOUT = 1, NIO = 0, N1D = 0, RZ = 4, RY = 4, RX = 4, RZR = 4;
+    static constexpr bool SPLIT_YZ = false;  // one coefficient for the y and z pair sums (yz)
     __host__ __device__ static constexpr int axis1d(int) { return 2; }
     __device__ __forceinline__ static void yz(double &acc, const SweepArgs &a, int r, double s) {
         acc = fma(a.s[r], s, acc);
@@ -75,6 +76,7 @@ struct Lap25Star {
 // Listing 1: B = a*A - (b*h2inv)*(6 neighbours - 6*A); scalars (h2inv, a, b)
 struct Jacobi7Star {
     static constexpr int R = 1, NIN = 1, NOUT = 1, NIO = 0, N1D = 0, RZ = 1, RY = 1, RX = 1, RZR = 1;
+    static constexpr bool SPLIT_YZ = false;
     __host__ __device__ static constexpr int axis1d(int) { return 2; }
     __device__ __forceinline__ static void yz(double &acc, const SweepArgs &, int, double s) { acc += s; }
     __device__ __forceinline__ static void x(double &acc, const SweepArgs &, int, double s) { acc += s; }
@@ -342,7 +344,12 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
                             // plane k+d (k = p-R) lives in slot (PH - R + d) mod NQ
                             const double zp = q[qs(PH, r)][py][px];
                             const double zm = q[qs(PH, -r)][py][px];
-                            B::yz(acc[py][px], a, r, (col[py + R + r][px] + col[py + R - r][px]) + (zp + zm));
+                            if constexpr (B::SPLIT_YZ) {  // distinct y and z coefficients (generated bodies)
+                                B::y(acc[py][px], a, r, col[py + R + r][px] + col[py + R - r][px]);
+                                B::z(acc[py][px], a, r, zp + zm);
+                            } else {
+                                B::yz(acc[py][px], a, r, (col[py + R + r][px] + col[py + R - r][px]) + (zp + zm));
+                            }
                         }
             }
             // x taps: the row window [cx-R, cx+2+R) lies in the aligned span
