@@ -29,13 +29,13 @@ def _plan(text):
     return p
 
 
-@settings(max_examples=300, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+@settings(max_examples=300, deadline=None, derandomize=True, suppress_health_check=[HealthCheck.too_slow])
 @given(st.text(alphabet=ALPHABET, max_size=300))
 def test_random_text_is_rejected_cleanly(text):
     _plan(text)
 
 
-@settings(max_examples=300, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+@settings(max_examples=300, deadline=None, derandomize=True, suppress_health_check=[HealthCheck.too_slow])
 @given(st.sampled_from(SPECS), st.integers(min_value=0, max_value=10 ** 6), st.sampled_from(["del", "dup", "sub"]),
        st.sampled_from(list("()[]{};,=+-*/0123456789kji.")))
 def test_mutated_specs_plan_or_fail_cleanly(spec, pos, op, ch):
@@ -49,7 +49,7 @@ def test_mutated_specs_plan_or_fail_cleanly(spec, pos, op, ch):
     _plan(text)
 
 
-@settings(max_examples=100, deadline=None)
+@settings(max_examples=100, deadline=None, derandomize=True)
 @given(st.sampled_from(SPECS), st.sampled_from(["maxfuse", "trivial"]))
 def test_fission_of_valid_specs_reparses(spec, kind):
     try:
