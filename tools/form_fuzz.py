@@ -66,37 +66,42 @@ stencil bx (out, A, s0, s1, s2) {{
 """, "jitbox_"
 
 
-n = int(sys.argv[1]) if len(sys.argv) > 1 else 30
-fails = runs = 0
-for seed in range(n):
-    rnd = random.Random(1000 + seed)
-    text, prefix = (star_spec if seed % 2 == 0 else box_spec)(rnd)
-    R = 4
-    dims = (2 * R + 3 + rnd.randrange(10), 2 * R + 5 + rnd.randrange(20), 2 * R + 20 + 2 * rnd.randrange(20))
-    try:
-        p0 = sdag.Plan(text, dims)
-    except sdag.SdagError as e:
-        print("plan error", seed, e)
-        fails += 1
-        continue
-    forms = [v for v in p0.variants() if v.startswith(prefix)]
-    if not forms:
-        print("FORM NOT DETECTED", seed, prefix, p0.variants()[:3])
-        fails += 1
-        continue
-    g = np.random.default_rng(seed)
-    A = g.uniform(-1, 1, dims)
-    sc = {"s0": 0.7, "s1": -0.4, "s2": 1.3}
-    for v in forms:
-        runs += 1
+def main():
+    n = int(sys.argv[1]) if len(sys.argv) > 1 else 30
+    fails = runs = 0
+    for seed in range(n):
+        rnd = random.Random(1000 + seed)
+        text, prefix = (star_spec if seed % 2 == 0 else box_spec)(rnd)
+        R = 4
+        dims = (2 * R + 3 + rnd.randrange(10), 2 * R + 5 + rnd.randrange(20), 2 * R + 20 + 2 * rnd.randrange(20))
         try:
-            plan = sdag.Plan(text, dims, variant=v)
-            dev = [torch.full(dims, float("nan"), dtype=torch.float64, device="cuda"), torch.from_numpy(A).cuda()]
-            plan.apply(dev, [], [sc["s0"], sc["s1"], sc["s2"]])
-            torch.cuda.synchronize()
-            compare(text, dims, {"A": A}, sc, {"out": dev[0].cpu().numpy(), "A": A})
-        except Exception as e:  # noqa: BLE001
+            p0 = sdag.Plan(text, dims)
+        except sdag.SdagError as e:
+            print("plan error", seed, e)
             fails += 1
-            print("FAIL", seed, v, dims, type(e).__name__, str(e)[:300], flush=True)
-print(f"form fuzz: {n} DAGs, {runs} variant runs, {fails} failures")
-sys.exit(1 if fails else 0)
+            continue
+        forms = [v for v in p0.variants() if v.startswith(prefix)]
+        if not forms:
+            print("FORM NOT DETECTED", seed, prefix, p0.variants()[:3])
+            fails += 1
+            continue
+        g = np.random.default_rng(seed)
+        A = g.uniform(-1, 1, dims)
+        sc = {"s0": 0.7, "s1": -0.4, "s2": 1.3}
+        for v in forms:
+            runs += 1
+            try:
+                plan = sdag.Plan(text, dims, variant=v)
+                dev = [torch.full(dims, float("nan"), dtype=torch.float64, device="cuda"), torch.from_numpy(A).cuda()]
+                plan.apply(dev, [], [sc["s0"], sc["s1"], sc["s2"]])
+                torch.cuda.synchronize()
+                compare(text, dims, {"A": A}, sc, {"out": dev[0].cpu().numpy(), "A": A})
+            except Exception as e:  # noqa: BLE001
+                fails += 1
+                print("FAIL", seed, v, dims, type(e).__name__, str(e)[:300], flush=True)
+    print(f"form fuzz: {n} DAGs, {runs} variant runs, {fails} failures")
+    return 1 if fails else 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())
