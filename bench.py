@@ -1,21 +1,35 @@
 #!/usr/bin/env python3
-"""bench.py -- headline benchmark of the sdag hot path on B200.
+"""bench.py -- the BASELINE benchmark of the sdag hot path on B200.
 
-Workload (BASELINE.json configs[1]): 25-point radius-4 FP64 Laplacian,
-512^3 grid per GPU, one sweep per step.  At N GPUs the grid is weak-scaled
-as z-slabs (512N x 512 x 512) with a per-step NCCL halo exchange (a7).
-A step = parse/plan done once up front (a1-a3, host), then one sweep
-(a4-a5) [+ exchange (a7) for N>1] over the resident input.
+BASELINE.json metric: "FP64 GFLOP/s and HBM GB/s per stencil, % of roofline,
+at 1/2/4/8 B200".  One JSON line (rank 0):
 
-Prints ONE JSON line (rank 0).  --impl reference times the CPU oracle (the
-reference arm of this tier) on the same metric/config.  --config selects
-another BASELINE stencil for reporting (not the headline line).
+  headline  (`value`, `roofline`, `e2e`, `cpu_baseline`): configs[1], the
+            25-point radius-4 FP64 Laplacian on a 512^3 grid per GPU, one
+            sweep per step (a4-a5 over inputs resident in HBM).  At N GPUs the
+            grid is weak-scaled as z-slabs (512N x 512 x 512) with the per-sweep
+            NCCL halo exchange (a7) inside the step.
+  per_config (N = 1): every other BASELINE stencil in the same run -- 1 (64^3
+            single sweep: latency), 1b (128 x 64^3 batched), 3 hypterm 320^3,
+            4 rhs4center 320^3, 5 the iterated 27-point smoother 1024^3 x 12
+            sweeps -- each with its own roofline, kernel time, traffic, clocks.
+  per_config (N > 1): config 5 as z-slabs (1024^3 per GPU, T = 12, NCCL
+            halo) with its weak-scaling efficiency E(N) = t_sweep(1) / t_sweep(N),
+            t_sweep(1) measured in the same run on each rank's own GPU.
+
+--gpus N without torchrun re-launches itself under torch.distributed.run with
+N ranks (127.0.0.1); under torchrun WORLD_SIZE must equal N.
+--impl reference times the CPU oracle (this tier's reference arm) on the
+headline workload with an identical `config`.
+Inputs: the synth/ recipes (counter-based generator), built on the device for
+the BASELINE sizes -- the same values the parity tests feed the oracle.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -28,38 +42,66 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 
 METRIC = "FP64 GFLOP/s and HBM GB/s per stencil, % of roofline, at 1/2/4/8 B200"
-
-CONFIGS = {
-    # name: (spec, dims per GPU, BASELINE config string, flops/pt)
-    "lap25": ("lap25", (512, 512, 512), "3D 4th-order 25-point Laplacian (order 4), 512^3 FP64, single GPU"),
-    "jacobi7": ("jacobi7", (64, 64, 64), "3D 7-point Jacobi (order 1), 64^3 FP64 grid, single sweep, 1 input/1 output"),
-    "hypterm": ("hypterm", (320, 320, 320), "ExpCNS hypterm-style DAG (order 4, ~8 inputs, multiple outputs), 320^3 FP64"),
-    "rhs4center": ("rhs4center", (320, 320, 320),
-                   "SW4 rhs4th3fort-style elastic-wave stencil (order 2, multi-statement, ~300 FLOP/pt), 320^3 FP64"),
-    "smooth27": ("smooth27", (1024, 1024, 1024),
-                 "iterated 27-point order-2 stencil, 1024^3 FP64 weak-scaled as z-slabs with halo exchange"),
+WORKLOAD = {
+    "1": "3D 7-point Jacobi (order 1), 64^3 FP64 grid, single sweep, 1 input/1 output",
+    "1b": "3D 7-point Jacobi (order 1), 64^3 FP64 grid, single sweep, batched: 128 independent problems per launch",
+    "2": "3D 4th-order 25-point Laplacian (order 4), 512^3 FP64, single GPU",
+    "3": "ExpCNS hypterm-style DAG (order 4, ~8 inputs, multiple outputs), 320^3 FP64",
+    "4": "SW4 rhs4th3fort-style elastic-wave stencil (order 2, multi-statement, ~300 FLOP/pt), 320^3 FP64",
+    "5": "iterated 27-point order-2 stencil, 1024^3 FP64 weak-scaled as z-slabs with halo exchange at 2/4/8 B200",
+}
+# config -> (stencil, dims per GPU, batch, sweeps per step)
+CONFIGS = {"1": ("jacobi7", (64, 64, 64), 1, 1), "1b": ("jacobi7", (64, 64, 64), 128, 1),
+           "2": ("lap25", (512, 512, 512), 1, 1), "3": ("hypterm", (320, 320, 320), 1, 1),
+           "4": ("rhs4center", (320, 320, 320), 1, 1), "5": ("smooth27", (1024, 1024, 1024), 1, 12)}
+# P100 numbers the paper prints, quoted as context (other hardware: never the target)
+PAPER_P100 = {
+    "3": {"value": 1.08e10 / 1e9, "unit": "GFLOP (per sweep, nvprof)", "note": "Table III P:1939 hypterm: 1.08e10 "
+          "FP64 flops per sweep at 312^3 interior; best P100 variant (global memory, P:2167-2173)"},
+    "4": {"value": 1.93e10 / 1e9, "unit": "GFLOP (per sweep, nvprof)", "note": "Table III P:1949 rhs4center: "
+          "1.93e10 executed FP64 flops per sweep (nvcc CSE; 666 x 316^3 = 2.10e10 canonical)"},
 }
 
+
+def headline_config(world):
+    """`config` of the headline line -- identical in both arms (same_config)."""
+    n = 512
+    return {"workload": WORKLOAD["2"], "stencil": "lap25", "grid_per_gpu": [n, n, n], "global_grid": [n * world, n, n],
+            "decomposition": f"z-slabs x{world}" if world > 1 else "none",
+            "l2": "input 1 GiB/GPU > 126 MB L2 (no flush needed)"}
+
+
+# ---------------------------------------------------------------------------
+# peaks, committed ncu counters, clocks
+# ---------------------------------------------------------------------------
 
 def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
         with open(p) as f:
             d = json.load(f)
-        return d.get("hbm_gbs", 6650.0), "measured"
-    return 6650.0, "fallback"
+        if "hbm_gbs" in d:
+            return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json copy bandwidth)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
 
 
-def load_traffic(variant, dims, batch=1):
-    """DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum) from a
-    committed ncu --set full capture of this variant at this size, else None."""
-    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if not os.path.exists(p):
-        return None
-    with open(p) as f:
-        d = json.load(f)
+def load_counters(variant, dims, batch=1):
+    """Per-launch ncu counters of this variant at this size, from one committed
+    `ncu --set full` capture (profiles/ncu_counters.json): DRAM bytes read+write
+    and executed FP64 flops (2 x DFMA + DADD + DMUL thread instructions)."""
     key = variant + "@" + "x".join(str(x) for x in ([batch] if batch > 1 else []) + list(dims))
-    return d.get(key)
+    out = {}
+    for fn in ("ncu_counters.json", "ncu_traffic.json"):
+        p = os.path.join(ROOT, "profiles", fn)
+        if os.path.exists(p):
+            with open(p) as f:
+                d = json.load(f).get(key)
+            if isinstance(d, dict):
+                for k, v in d.items():
+                    out.setdefault(k, v)
+            elif d is not None:
+                out.setdefault("dram_bytes", d)
+    return out
 
 
 class Clocks:
@@ -77,7 +119,7 @@ class Clocks:
              "clocks_event_reasons.sw_power_cap")
         try:
             p = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={q}", "--format=csv,noheader,nounits",
-                                  "-lms", "100"], stdout=subprocess.PIPE, text=True)
+                                  "-lms", "50"], stdout=subprocess.PIPE, text=True)
         except Exception:
             return
         while not self._stop.is_set():
@@ -105,7 +147,7 @@ class Clocks:
         if not self.samples:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
-        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if len(s) > 1 and s[1].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = set()
         for s in self.samples:
@@ -116,267 +158,325 @@ class Clocks:
                 "reasons": sorted(reasons), "samples": len(self.samples)}
 
 
-def cpu_baseline_lap25(A, c, seconds=10.0):
-    """Time the oracle (as it stands) on the same 512^3 input: whole sweeps,
-    repeated for ~`seconds` of CPU work (the bounded sample)."""
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
+# ---------------------------------------------------------------------------
+# device inputs (synth recipes, bit-identical to the parity tests' arrays)
+# ---------------------------------------------------------------------------
+
+def build_arrays(sdag, plan, name, dims, batch=1):
+    """3D formals in formal order (inputs/inouts from the recipe, outputs empty),
+    1D formals, scalars in formal order."""
+    import torch
+    import synth
+    cfg, a3, a1, sc = synth.recipe(name)
+    shape = (batch, *dims) if batch > 1 else tuple(dims)
+    arrays3d, arrays1d, scal = [], [], []
+    for kind, _, nm, role in plan.args():
+        if kind == 0:
+            if nm in a3:
+                lo, hi = a3[nm]
+                arrays3d.append(synth.uniform_torch(shape, lo, hi, cfg, nm))
+            else:
+                arrays3d.append(torch.empty(shape, dtype=torch.float64, device="cuda"))
+        elif kind == 1:
+            lo, hi = a1[nm]
+            n = dims[role]
+            arrays1d.append(torch.from_numpy(synth.uniform((n,), lo, hi, cfg, nm)).cuda())
+        else:
+            scal.append(sc[nm])
+    return arrays3d, arrays1d, scal
+
+
+def timed(step, steps, warmup, stream, clock_index):
+    """W untimed steps, then K steps between CUDA events on `stream` (synchronised
+    on both sides), nvidia-smi clocks sampled during the timed region.
+    -> (ms per step, launches per step, clocks)"""
+    import torch
+    import paper_conf_ipps_rawatvsrps19_b200 as sdag
+    for _ in range(warmup):
+        step()
+    torch.cuda.synchronize()
+    l0 = sdag.launch_count()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with Clocks(clock_index) as clk:
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(steps):
+            step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / steps, (sdag.launch_count() - l0) / steps, clk.summary()
+
+
+def roofline(info, kms, batch, peak_hbm, peak_src, fp64_peak, counters, kernel, sweeps_per_launch=1):
+    """The kernel's roofline on ALGORITHMIC work per launch (DESIGN.md 6.3:
+    bytes = R10, flops = R9 over the interior points one launch writes)."""
+    pts = info["points"] * batch
+    alg_bytes = info["bytes_per_point"] * pts
+    canon = info["flops_per_point"] * pts * sweeps_per_launch
+    t = kms * 1e-3
+    hbm_bound = alg_bytes / (peak_hbm * 1e9)
+    exe = counters.get("fp64_flops")
+    F = min(canon, exe) if exe else canon
+    fp_bound = F / fp64_peak if fp64_peak else 0.0
+    r = {"kernel": kernel, "kernel_ms": kms, "traffic": counters.get("dram_bytes"),
+         "alg_bytes_per_launch": alg_bytes, "canonical_flops_per_launch": canon,
+         "executed_fp64_flops_per_launch": exe}
+    if fp_bound > hbm_bound:  # FP64-pipe bound (rhs4center): "alu" per the contract, the FP64 pipe's DFMA peak
+        r.update({"bound": "alu", "pipe": "fp64", "achieved": F / t / 1e12, "peak": fp64_peak / 1e12,
+                  "unit": "TFLOP/s", "frac": fp_bound / t, "frac_canonical_flops": (canon / fp64_peak) / t,
+                  "peak_source": "measured DFMA rate (sdag_measure_fp64_peak, all SMs, this run); "
+                                 "nominal 148 SM x 64 DFMA/clk x 2 x 1.965 GHz = 37.2 TFLOP/s",
+                  "F": "min(canonical, ncu-executed) flops (SURVEY 8(d))" if exe else "canonical flops"})
+    else:
+        r.update({"bound": "hbm", "achieved": alg_bytes / t / 1e9, "peak": peak_hbm, "unit": "GB/s",
+                  "frac": hbm_bound / t, "peak_source": peak_src})
+    return r
+
+
+# ---------------------------------------------------------------------------
+# per-config measurements (N = 1)
+# ---------------------------------------------------------------------------
+
+def measure_config(cid, steps, warmup, peak_hbm, peak_src, fp64_peak, tune=False):
+    import torch
+    import paper_conf_ipps_rawatvsrps19_b200 as sdag
+    name, dims, batch, T = CONFIGS[cid]
+    plan = sdag.Plan(sdag.spec_text(name), dims, batch=batch, tune=tune)
+    info = plan.info
+    arrays3d, arrays1d, scal = build_arrays(sdag, plan, name, dims, batch)
+    stream = torch.cuda.current_stream()
+    res = {"workload": WORKLOAD[cid], "stencil": name, "grid": list(dims), "batch": batch, "sweeps_per_step": T,
+           "variant": info["variant"], "flops_per_point": info["flops_per_point"],
+           "bytes_per_point": info["bytes_per_point"]}
+    if cid == "1":
+        # one 2 MB problem: latency-bound (launch + one short z-stream); L2 flushed
+        # between iterations, each launch timed alone with events
+        flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+        ev = []
+        for it in range(warmup + steps):
+            flush.fill_(it & 0xFF)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            plan.apply(arrays3d, arrays1d, scal, stream=stream)
+            b.record(stream)
+            ev.append((a, b))
+        torch.cuda.synchronize()
+        times = [a.elapsed_time(b) for a, b in ev[warmup:]]
+        ms = statistics.median(times)
+        res.update({"ms_per_step": ms, "us_min": min(times) * 1e3, "launches_per_step": 1,
+                    "l2": "flushed (256 MB write) before every timed launch",
+                    "gflops": info["flops_per_point"] * info["points"] / (ms * 1e-3) / 1e9,
+                    "note": "latency, not throughput: 2 MB of traffic cannot fill 148 SMs (SURVEY 8(d) note)",
+                    "kernel": plan.kernel_name(1)})
+        return res
+    if T > 1:
+        b0, b1 = arrays3d[[r[3] for r in plan.args() if r[0] == 0].index(0)], None
+        b1 = b0.clone()
+
+        def step():
+            plan.apply_iterated(b0, b1, T, scal, stream=stream)
+    elif batch > 1:
+        def step():
+            plan.apply_batched(batch, arrays3d, arrays1d, scal, stream=stream)
+    else:
+        def step():
+            plan.apply(arrays3d, arrays1d, scal, stream=stream)
+    ms, lps, clk = timed(step, steps, warmup, stream, torch.cuda.current_device())
+    kms = ms / lps
+    spl = T / lps  # sweeps per launch
+    if spl > 1:
+        kernel = plan.kernel_name(int(round(spl))) if abs(spl - round(spl)) < 1e-9 else plan.kernel_name(2)
+        variant = [ln for ln in plan.describe().splitlines() if "temporal fusion" in ln]
+        variant = variant[0].split(":", 1)[1].split()[0] if variant else info["variant"]
+    else:
+        kernel, variant = plan.kernel_name(1), info["variant"]
+    counters = load_counters(variant, dims, batch)
+    pts_step = info["points"] * batch * T
+    res.update({"variant": variant, "ms_per_step": ms, "launches_per_step": lps,
+                "gflops": info["flops_per_point"] * pts_step / (ms * 1e-3) / 1e9,
+                "hbm_gbs": info["bytes_per_point"] * pts_step / (ms * 1e-3) / 1e9,
+                "roofline": roofline(info, kms, batch, peak_hbm, peak_src, fp64_peak, counters, kernel, spl),
+                "clocks": clk, "l2": "inputs > 126 MB L2 (no flush needed)"})
+    if spl > 1:
+        # temporal fusion (NEXT-1): a launch reads and writes HBM once for spl
+        # sweeps, so per sweep it can beat the unfused roofline
+        res["roofline"]["sweep_equivalent"] = {"sweeps_per_launch": spl,
+                                               "frac_of_unfused_roofline": res["roofline"]["frac"] * spl}
+    if cid in PAPER_P100:
+        res["paper_p100_context"] = PAPER_P100[cid]
+    del arrays3d, arrays1d
+    torch.cuda.empty_cache()
+    return res
+
+
+# ---------------------------------------------------------------------------
+# the CPU oracle (cpu_baseline leg and the reference arm)
+# ---------------------------------------------------------------------------
+
+def oracle_lap25_throughput(A, c, seconds, groups=3):
+    """The oracle as it stands on the host cores: whole 512^3 sweeps of the
+    benchmark input, `groups` timed batches of ~seconds/groups each; the best
+    batch is the value (min of 3)."""
     import oracle
-    cores = len(os.sched_getaffinity(0))
     nz, ny, nx = A.shape
     out = np.zeros_like(A)
-    oracle.lap25(A, c, out=out, krange=(4, 6))  # warm (build + page-in)
-    reps, t0 = 0, time.perf_counter()
-    while True:
-        oracle.lap25(A, c, out=out)
-        reps += 1
-        if time.perf_counter() - t0 >= seconds:
-            break
-    dt = time.perf_counter() - t0
-    pts = reps * (nz - 8) * (ny - 8) * (nx - 8)
-    return {"value": pts * 29 / dt / 1e9, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
-            "sample": f"{reps} full 512^3 sweeps of the benchmark input ({pts} interior points), {dt:.1f} s, "
-                      f"OpenMP over k with {cores} threads"}
+    oracle.lap25(A, c, out=out, krange=(4, 6))  # build + page-in
+    oracle.lap25(A, c, out=out)  # warm
+    rates, reps_total, t_total = [], 0, 0.0
+    for _ in range(groups):
+        reps, t0 = 0, time.perf_counter()
+        while True:
+            oracle.lap25(A, c, out=out)
+            reps += 1
+            if time.perf_counter() - t0 >= seconds / groups:
+                break
+        dt = time.perf_counter() - t0
+        rates.append(reps * (nz - 8) * (ny - 8) * (nx - 8) * 29 / dt / 1e9)
+        reps_total += reps
+        t_total += dt
+    return max(rates), reps_total, t_total
+
+
+def cpu_cores():
+    n = len(os.sched_getaffinity(0))
+    omp = os.environ.get("OMP_NUM_THREADS")
+    return min(n, int(omp)) if omp and omp.isdigit() else n
 
 
 def run_reference(args):
     """--impl reference: the CPU oracle (this tier's reference arm) on the host
-    cores, same metric and config: each step is one full 512^3 sweep of the same
-    seeded input (~0.1-0.3 s of CPU work per step)."""
-    rank = int(os.environ.get("RANK", "0"))
-    if rank != 0:
+    cores, same metric and config; each step one full 512^3 sweep of the same
+    seeded input.  Rank 0 only."""
+    if int(os.environ.get("RANK", "0")) != 0:
         return 0
+    import oracle
     import synth
-    dims = CONFIGS["lap25"][1]
-    ins, sc = synth.lap25_inputs(dims, cfg="cfg2")
+    ins, sc = synth.lap25_inputs((512, 512, 512), cfg="cfg2")
     A = ins["A"]
     c = [sc[k] for k in ("c0", "c1", "c2", "c3", "c4")]
-    import oracle
-    cores = len(os.sched_getaffinity(0))
     out = np.zeros_like(A)
-    nz, ny, nx = dims
     oracle.lap25(A, c, out=out, krange=(4, 6))
     for _ in range(args.warmup):
         oracle.lap25(A, c, out=out)
-    t0 = time.perf_counter()
+    times = []
     for _ in range(args.steps):
+        t0 = time.perf_counter()
         oracle.lap25(A, c, out=out)
-    dt = time.perf_counter() - t0
-    pts = args.steps * (nz - 8) * (ny - 8) * (nx - 8)
+        times.append(time.perf_counter() - t0)
+    dt = sum(times)
+    pts = args.steps * 504 ** 3
     val = pts * 29 / dt / 1e9
-    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "GFLOP/s", "n_gpus": args.gpus,
+    world = int(os.environ.get("WORLD_SIZE", str(args.gpus)))
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "GFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": CONFIGS["lap25"][2], "stencil": "lap25", "grid": list(dims),
-                       "step": "one full oracle sweep of the 512^3 input on the host cores"},
-            "cpu_baseline": {"value": val, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
-                             "sample": f"{args.steps} full 512^3 sweeps (all interior points)"},
+            "config": headline_config(1),
+            "cpu_baseline": {"value": val, "unit": "GFLOP/s", "cores": cpu_cores(), "kind": "oracle",
+                             "cpu_model": cpu_model(), "best_step_gflops": 504 ** 3 * 29 / min(times) / 1e9,
+                             "sample": f"{args.steps} full 512^3 sweeps of the benchmark input (all {504 ** 3} "
+                                       f"interior points each), OpenMP over k"},
             "e2e": {"value": val, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line))
     return 0
 
 
-def run_other(args):
-    """One line for another BASELINE stencil at N=1 (recorded under profiles/, not the headline).
-    Inputs: seeded torch generator on the device (timing is data-independent; parity of
-    the same kernels on synth/ inputs is in tests/test_gpu_parity.py)."""
+# ---------------------------------------------------------------------------
+# multi-GPU: config 5 as z-slabs (the BASELINE weak-scaling workload)
+# ---------------------------------------------------------------------------
+
+def measure_config5_slabs(tdist, rank, world, local, steps, warmup, comm, halo="nccl"):
+    """Config 5 per rank: 1024^3 owned planes, T = 12, ghost depth 2 (one NCCL
+    exchange per fused 2-sweep launch, overlapped with the interior launch);
+    plus t_sweep(1): the same 1024^3 iteration on this GPU alone (single-GPU
+    plan), so E(N) = t_sweep(1) / t_sweep(N) comes from one run."""
     import torch
     import paper_conf_ipps_rawatvsrps19_b200 as sdag
-    name = args.config
-    spec = sdag.spec_text(name)
-    dims = CONFIGS[name][1]
-    torch.cuda.set_device(0)
-    g = torch.Generator(device="cuda").manual_seed(20190520)
-    batch, T = 1, 1
-    if name == "jacobi7":
-        batch = 128  # config 1b: 128 independent 64^3 problems in one launch (latency-bound alone)
-    # the non-headline lines use the measured (hierarchical tune=1) plan, as a
-    # production user would; plan time is outside the timed region
-    plan = sdag.Plan(spec, dims, batch=batch, tune=not args.no_tune, variant=args.variant)
-    info = plan.info
-    shape = (batch, *dims) if batch > 1 else dims
-    scal = {"jacobi7": [4.0, 0.5, 0.25], "hypterm": [0.5, 0.25, 0.125, 0.8, -0.2, 4 / 105, -1 / 280],
-            "rhs4center": [0.75, 1 / 6, 1 / 144, 1.0, 1.0], "smooth27": [-128 / 30, 14 / 30, 3 / 30, 1 / 30, 0.125]}[name]
-    arrs = [torch.rand(shape, dtype=torch.float64, device="cuda", generator=g) + 0.5
-            for _ in range(info["n_arrays3d"])]
-    a1 = [torch.rand(dims[2 - q], dtype=torch.float64, device="cuda", generator=g) + 0.5
-          for q in range(info["n_arrays1d"])]
-    if name == "smooth27":
-        T = 12  # config 5: iterated T = 12 sweeps (Table I "T", reading R5)
-        b0, b1 = arrs[1], arrs[0]
-
-        def step():
-            plan.apply_iterated(b0, b1, T, scal)
-    elif batch > 1:
-        def step():
-            plan.apply_batched(batch, arrs, a1, scal)
-    else:
-        def step():
-            plan.apply(arrs, a1, scal)
-    for _ in range(args.warmup):
-        step()
-    torch.cuda.synchronize()
-    l0 = sdag.launch_count()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with Clocks(0) as clk:
-        torch.cuda.synchronize()
-        e0.record()
-        for _ in range(args.steps):
-            step()
-        e1.record()
-        torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1) / args.steps
-    launches = sdag.launch_count() - l0
-    pts = info["points"] * batch * T
-    flops = info["flops_per_point"] * pts
-    byts = info["bytes_per_point"] * pts
-    kms = ms / (launches / args.steps)
-    hbm, src = load_peaks()
-    if name == "rhs4center":
-        fp64 = sdag.fp64_peak()
-        achieved = info["flops_per_point"] * info["points"] / (kms * 1e-3) / 1e12
-        roof = {"bound": "fp64", "achieved": achieved, "peak": fp64 / 1e12, "unit": "TFLOP/s", "frac": achieved * 1e12 / fp64,
-                "peak_source": "measured DFMA micro-benchmark (sdag_measure_fp64_peak) in this run"}
-    else:
-        achieved = info["bytes_per_point"] * info["points"] * batch / (kms * 1e-3) / 1e9
-        roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
-                "peak_source": src}
-    kernel = info["variant"]
-    if name == "smooth27" and launches < T * args.steps:
-        # temporal fusion (NEXT-1): the launches are 2-sweep kernels; one launch
-        # reads its input and writes its output once, so its algorithmic bytes
-        # are one sweep's -- the roofline below is the fused kernel's own
-        fl = [ln for ln in plan.describe().splitlines() if "temporal fusion" in ln]
-        kernel = fl[0].split(":", 1)[1].split()[0] if fl else kernel
-        # per SURVEY 8(d)'s unit (one written point of one sweep): a launch processes
-        # T / launches sweeps' units, so the sweep-equivalent rate can exceed the
-        # HBM roofline of unfused sweeps -- the point of temporal fusion
-        spl = T * args.steps / launches
-        roof["sweep_equivalent"] = {"sweeps_per_launch": spl, "achieved": achieved * spl,
-                                    "frac": achieved * spl / hbm}
-    roof.update({"traffic": load_traffic(kernel, dims, batch), "kernel_ms": kms, "kernel": kernel})
-    line = {"metric": METRIC, "value": flops / (ms * 1e-3) / 1e9, "unit": "GFLOP/s", "n_gpus": 1,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded torch generator)",
-            "config": {"workload": CONFIGS[name][2], "stencil": name, "grid": list(dims), "batch": batch,
-                       "sweeps_per_step": T, "variant": kernel, "tuned": not args.no_tune,
-                       "l2": "inputs > 126 MB L2 (no flush needed)",
-                       "launches_per_step": launches // args.steps, "flops_per_point": info["flops_per_point"],
-                       "bytes_per_point": info["bytes_per_point"]},
-            "hbm_gbs": byts / (ms * 1e-3) / 1e9, "roofline": roof, "gpu_launches": launches,
-            "clocks": clk.summary()}
-    print(json.dumps(line))
-    return 0
-
-
-def run_slabs27(args):
-    """Config 5 as BASELINE names it: the iterated 27-point smoother, 1024^3 per
-    GPU, T = 12 sweeps per step, weak-scaled as z-slabs (one rank per GPU).
-    --halo nccl: ghost planes exchanged by NCCL send/recv on a comm stream,
-    overlapped with the interior launch (sdag_dist_apply_iterated);
-    --halo p2p: the boundary launches store their planes straight into the
-    neighbours' ghost planes over NVLink (sdag_dist_p2p_apply_iterated; CUDA IPC
-    handles exchanged over the process group), no NCCL.  Ghost depth 2 R_z
-    (time_tile 2): one exchange per fused 2-sweep launch.
-    SDAG_BENCH_SAME_DEVICE=1 maps every rank to cuda:0 (plumbing check of the
-    multi-process p2p path on one GPU; times are then not scaling numbers)."""
-    import torch
-    import torch.distributed as tdist
-    import paper_conf_ipps_rawatvsrps19_b200 as sdag
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = 0 if os.environ.get("SDAG_BENCH_SAME_DEVICE") else int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    halo = args.halo or "nccl"
-    pg = None
-    if world > 1:
-        if halo == "p2p":
-            tdist.init_process_group("gloo")  # host plumbing only: IPC handles, barrier, timing reduce
-        else:
-            tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        pg = tdist
-    name, T, tt = "smooth27", 12, 2
-    spec = sdag.spec_text(name)
-    n = int(os.environ.get("SDAG_BENCH_SLAB_N", "1024"))
+    import synth
+    n, T, tt = 1024, 12, 2
+    spec = sdag.spec_text("smooth27")
+    cfg, a3, _, sc = synth.recipe("smooth27")
+    scal = [sc[k] for k in ("w0", "w1", "w2", "w3", "nu")]
+    stream = torch.cuda.current_stream()
+    # single-GPU reference time on this rank's device (no communication)
+    plan1 = sdag.Plan(spec, (n, n, n))
+    b0 = synth.uniform_torch((n, n, n), -1.0, 1.0, cfg, "A")
+    b1 = b0.clone()
+    ms1, _, _ = timed(lambda: plan1.apply_iterated(b0, b1, T, scal, stream=stream), steps, warmup, stream, local)
+    del b0, b1, plan1
+    torch.cuda.empty_cache()
     gdims = (n * world, n, n)
-    scal = [-128 / 30, 14 / 30, 3 / 30, 1 / 30, 0.125]
-    comm = None
-    if halo == "nccl" and world > 1:
-        uid = [sdag.nccl_unique_id() if rank == 0 else None]
-        tdist.broadcast_object_list(uid, src=0)
-        comm = sdag.nccl_comm_create(uid[0], world, rank, local)
-    dd = sdag.Dist(spec, gdims, rank, world, comm=comm, time_tile=tt, variant=args.variant)
+    dd = sdag.Dist(spec, gdims, rank, world, comm=comm, time_tile=tt)
     (nza, ny, nx), g0 = dd.layout()
     part = sdag.slab_partition2(gdims[0], 1, tt, world, rank)
-    stream = torch.cuda.current_stream()
-    full = torch.from_numpy(__import__("synth").uniform((nza, ny, nx), -1.0, 1.0, "cfg5-slab", rank))
+    x0 = synth.uniform_torch((nza, ny, nx), -1.0, 1.0, cfg + "-slab", rank)
     if halo == "p2p":
-        b0, b1 = dd.p2p_alloc()
-        b0.copy_(full)
-        b1.copy_(full)
+        # the boundary launches store their planes straight into the neighbours'
+        # ghost planes over NVLink (CUDA IPC), flag-ordered -- no NCCL step
+        p0, _ = dd.p2p_alloc()
+        p0.copy_(x0)
+        x0 = p0
+        hs = [None] * world
+        tdist.all_gather_object(hs, dd.p2p_handle())
+        if rank > 0:
+            dd.p2p_attach(0, hs[rank - 1])
+        if rank < world - 1:
+            dd.p2p_attach(1, hs[rank + 1])
         torch.cuda.synchronize()
-        if world > 1:
-            hs = [None] * world
-            tdist.all_gather_object(hs, dd.p2p_handle())
-            if rank > 0:
-                dd.p2p_attach(0, hs[rank - 1])
-            if rank < world - 1:
-                dd.p2p_attach(1, hs[rank + 1])
-
-        def step():
-            dd.p2p_apply_iterated(T, scalars=scal, stream=stream)
+        step = lambda: dd.p2p_apply_iterated(T, scalars=scal, stream=stream)  # noqa: E731
     else:
-        b0 = full.cuda()
-        b1 = b0.clone()
+        x1 = x0.clone()
         cs = torch.cuda.Stream()
-
-        def step():
-            dd.apply_iterated(b0, b1, T, scalars=scal, stream=stream, comm_stream=cs)
-    del full
+        step = lambda: dd.apply_iterated(x0, x1, T, scalars=scal, stream=stream, comm_stream=cs)  # noqa: E731
+    tdist.barrier()
+    msN, lps, clk = timed(step, steps, warmup, stream, local)
+    t = torch.tensor([ms1, msN], dtype=torch.float64, device="cuda")
+    tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+    ms1m, msNm = float(t[0]), float(t[1])
+    pts = torch.tensor([float((part["k_hi"] - part["k_lo"]) * (ny - 2) * (nx - 2) * T)], dtype=torch.float64,
+                       device="cuda")
+    tdist.all_reduce(pts, op=tdist.ReduceOp.SUM)
     info = dd.plan.info
-    pts_rank = (part["k_hi"] - part["k_lo"]) * (ny - 2) * (nx - 2) * T
-    for _ in range(args.warmup):
-        step()
-    torch.cuda.synchronize()
-    if pg:
-        tdist.barrier()
-    l0 = sdag.launch_count()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with Clocks(local) as clk:
-        torch.cuda.synchronize()
-        e0.record(stream)
-        for _ in range(args.steps):
-            step()
-        e1.record(stream)
-        torch.cuda.synchronize()
-    launches = sdag.launch_count() - l0
-    ms = e0.elapsed_time(e1)
-    red = torch.tensor([ms, float(pts_rank)], dtype=torch.float64)
-    if pg:
-        tdist.barrier()
-        mx = red.clone()
-        tdist.all_reduce(mx, op=tdist.ReduceOp.MAX)
-        sm = red.clone()
-        tdist.all_reduce(sm, op=tdist.ReduceOp.SUM)
-        ms_max, total_pts = float(mx[0]), float(sm[1])
-    else:
-        ms_max, total_pts = ms, float(pts_rank)
-    flops = total_pts * info["flops_per_point"] * args.steps
-    if rank == 0:
-        line = {"metric": METRIC, "value": flops / (ms_max * 1e-3) / 1e9, "unit": "GFLOP/s", "n_gpus": world,
-                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
-                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-                "data": "synthetic (counter-based generator, per-rank slab)",
-                "config": {"workload": CONFIGS[name][2], "stencil": name, "grid_per_gpu": [n, n, n],
-                           "global_grid": list(gdims), "decomposition": f"z-slabs x{world}", "halo": halo,
-                           "time_tile": tt, "sweeps_per_step": T, "variant": info["variant"],
-                           "same_device": bool(os.environ.get("SDAG_BENCH_SAME_DEVICE")),
-                           "l2": "8 GiB slab/GPU > 126 MB L2 (no flush needed)"},
-                "hbm_gbs_sweep_equivalent": total_pts * info["bytes_per_point"] * args.steps / (ms_max * 1e-3) / 1e9,
-                "gpu_launches": launches, "clocks": clk.summary()}
-        print(json.dumps(line))
-    if pg:
-        tdist.barrier()
-        tdist.destroy_process_group()
-    return 0
+    del x0, step
+    torch.cuda.empty_cache()
+    return {"workload": WORKLOAD["5"], "stencil": "smooth27", "grid_per_gpu": [n, n, n], "global_grid": list(gdims),
+            "decomposition": f"z-slabs x{world}",
+            "halo": ("nccl send/recv" if halo == "nccl" else "p2p stores fused into the boundary kernels")
+            + " (ghost depth 2: one exchange per fused 2-sweep launch)",
+            "sweeps_per_step": T, "ms_per_step": msNm, "ms_per_sweep": msNm / T,
+            "single_gpu_ms_per_sweep": ms1m / T, "weak_scaling_efficiency": ms1m / msNm,
+            "gflops": float(pts) * info["flops_per_point"] / (msNm * 1e-3) / 1e9,
+            "hbm_gbs_sweep_equivalent": float(pts) * info["bytes_per_point"] / (msNm * 1e-3) / 1e9,
+            "launches_per_step": lps, "clocks": clk}
+
+
+# ---------------------------------------------------------------------------
+# launcher
+# ---------------------------------------------------------------------------
+
+def free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def relaunch(args_ns):
+    """--gpus N without torchrun: run this script under torch.distributed.run."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args_ns.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 def main():
@@ -387,222 +487,190 @@ def main():
     ap.add_argument("--impl", default="sdag", choices=["sdag", "reference"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--variant", default=None)
-    ap.add_argument("--tune", action="store_true", help="headline: tune=1 plan (the --config lines tune by default)")
-    ap.add_argument("--no-tune", action="store_true", help="--config lines: heuristic plan instead of tune=1")
-    ap.add_argument("--force-dist", action="store_true",
-                    help="take the z-slab/NCCL path even on one rank (plumbing check of the multi-GPU code)")
-    ap.add_argument("--config", default="lap25", choices=list(CONFIGS),
-                    help="lap25 = the headline line; the others record the remaining BASELINE stencils (N=1)")
-    ap.add_argument("--halo", default=None, choices=["nccl", "p2p"],
-                    help="z-slab halo path (default nccl); with --config smooth27: the z-slab run of config 5 "
-                         "(BASELINE's multi-GPU workload)")
+    ap.add_argument("--no-per-config", action="store_true", help="headline only")
+    ap.add_argument("--configs", default="1,1b,3,4,5", help="per_config entries at N = 1")
+    ap.add_argument("--variant", default=None, help="force the headline plan's variant")
+    ap.add_argument("--tune", action="store_true", help="tune=1 plans (measured pick) instead of the heuristic")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--cpu-baseline-only", action="store_true", help=argparse.SUPPRESS)
+    ap.add_argument("--halo", default="nccl", choices=["nccl", "p2p"], help="N > 1: config 5's slab halo path")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
+    env_world = os.environ.get("WORLD_SIZE")
     if args.impl == "reference":
         return run_reference(args)
-    if args.config == "smooth27" and (args.halo or int(os.environ.get("WORLD_SIZE", "1")) > 1):
-        return run_slabs27(args)
-    if args.config != "lap25":
-        return run_other(args)
+    if args.cpu_baseline_only:
+        import synth
+        ins, _ = synth.lap25_inputs((512, 512, 512), cfg="cfg2")
+        c = [synth.LAP25_COEFS[k] for k in ("c0", "c1", "c2", "c3", "c4")]
+        val, reps, tt = oracle_lap25_throughput(ins["A"], c, args.cpu_seconds)
+        print(json.dumps({"value": val, "unit": "GFLOP/s", "cores": cpu_cores(), "kind": "oracle",
+                          "cpu_model": cpu_model(),
+                          "sample": f"{reps} full 512^3 sweeps of the benchmark input in 3 timed batches "
+                                    f"({tt:.1f} s); value = the best batch (min of 3); OpenMP over k, "
+                                    f"separate process"}))
+        return 0
+    if env_world is None and args.gpus > 1:
+        return relaunch(args)
+    world = int(env_world or "1")
+    if world != args.gpus:
+        print(f"bench: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
+        return 2
+    if world > 1:
+        # NCCL communicator init lines (nranks) visible to the driver
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
 
     import torch
     import paper_conf_ipps_rawatvsrps19_b200 as sdag
     import synth
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = 0 if os.environ.get("SDAG_BENCH_SAME_DEVICE") else int(os.environ.get("LOCAL_RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
-    p2p = args.halo == "p2p"
-    dist = None
+    tdist = None
+    comm = None
     if world > 1:
         import torch.distributed as tdist
-        if p2p:  # host plumbing only (IPC handles, barriers, the timing reduce)
-            tdist.init_process_group("gloo")
-        else:
-            tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        dist = tdist
-    red_dev = "cpu" if p2p else "cuda"
-    name = "lap25"
-    spec = sdag.spec_text(name)
-    ldims = CONFIGS[name][1]
-    gdims = (ldims[0] * world, ldims[1], ldims[2])
-    use_dist = world > 1 or args.force_dist or args.halo == "p2p"
-    ins, sc = synth.lap25_inputs(ldims, cfg="cfg2") if not use_dist else (None, dict(synth.LAP25_COEFS))
-    c = [sc[k] for k in ("c0", "c1", "c2", "c3", "c4")]
+        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        uid = [sdag.nccl_unique_id() if rank == 0 else None]
+        tdist.broadcast_object_list(uid, src=0)
+        comm = sdag.nccl_comm_create(uid[0], world, rank, local)
+    peak_hbm, peak_src = load_peaks()
     stream = torch.cuda.current_stream()
+    spec = sdag.spec_text("lap25")
+    n = 512
+    c = [synth.LAP25_COEFS[k] for k in ("c0", "c1", "c2", "c3", "c4")]
 
-    if not use_dist:
-        plan = sdag.Plan(spec, ldims, tune=args.tune, variant=args.variant)
-        A = ins["A"]
-        dA = torch.from_numpy(A).cuda()
-        dB = torch.zeros(ldims, dtype=torch.float64, device="cuda")
-        arrays = [dB, dA]
+    # ---- headline: config 2 ----
+    if world == 1:
+        plan = sdag.Plan(spec, (n, n, n), tune=args.tune, variant=args.variant)
         info = plan.info
-        pts_rank = info["points"]
+        dA = synth.uniform_torch((n, n, n), -1.0, 1.0, "cfg2", "A")
+        dB = torch.zeros((n, n, n), dtype=torch.float64, device="cuda")
 
         def step():
-            plan.apply(arrays, scalars=c, stream=stream)
+            plan.apply([dB, dA], scalars=c, stream=stream)
+        ms, lps, clk = timed(step, args.steps, args.warmup, stream, local)
+        kms = ms / lps
+        pts_total = info["points"]
+        kplan = plan
     else:
-        comm = None
-        if not p2p:
-            uid = [None]
-            if rank == 0:
-                try:
-                    uid = [sdag.nccl_unique_id()]
-                except sdag.SdagError as e:  # no usable NCCL: the peer-memory halo needs none
-                    print(f"bench: NCCL halo unavailable ({e}); using the p2p halo", file=sys.stderr)
-            if dist:
-                dist.broadcast_object_list(uid, src=0)
-            if uid[0] is None:
-                p2p = True
-            else:
-                comm = sdag.nccl_comm_create(uid[0], world, rank, local)
-        dd = sdag.Dist(spec, gdims, rank, world, comm=comm, tune=args.tune, variant=args.variant)
+        dd = sdag.Dist(spec, (n * world, n, n), rank, world, comm=comm, tune=args.tune, variant=args.variant)
         (nza, ny, nx), g0 = dd.layout()
-        part = sdag.slab_partition(gdims[0], 4, world, rank)
-        # this rank's slab of the global synthetic input, regenerated from the counter-based generator
-        full = synth.uniform((nza, ny, nx), -1.0, 1.0, "cfg2-slab", rank)
-        if p2p:
-            # --halo p2p: library-owned slab buffers; the input's ghost planes are
-            # pushed over NVLink by the neighbours and flag-ordered (one sweep =
-            # sdag_dist_p2p_apply_iterated with T = 1), no NCCL
-            dA, dB = dd.p2p_alloc()
-            dA.copy_(torch.from_numpy(full))
-            dB.zero_()
-            torch.cuda.synchronize()
-            if dist:
-                hs = [None] * world
-                dist.all_gather_object(hs, dd.p2p_handle())
-                if rank > 0:
-                    dd.p2p_attach(0, hs[rank - 1])
-                if rank < world - 1:
-                    dd.p2p_attach(1, hs[rank + 1])
-        else:
-            dA = torch.from_numpy(full).cuda()
-            dB = torch.zeros((nza, ny, nx), dtype=torch.float64, device="cuda")
-        arrays = [dB, dA]
-        plan = dd.plan
-        info = plan.info
-        pts_rank = (part["k_hi"] - part["k_lo"]) * (ny - 8) * (nx - 8)
-        comm_stream = torch.cuda.Stream()
+        part = sdag.slab_partition(n * world, 4, world, rank)
+        dA = synth.uniform_torch((nza, ny, nx), -1.0, 1.0, "cfg2-slab", rank)
+        dB = torch.zeros((nza, ny, nx), dtype=torch.float64, device="cuda")
+        cs = torch.cuda.Stream()
+        kplan = dd.plan
+        info = kplan.info
 
         def step():
-            if p2p:
-                dd.p2p_apply_iterated(1, scalars=c, stream=stream)
-            else:
-                dd.apply(arrays, scalars=c, stream=stream, comm_stream=comm_stream)
-
-    flops_pt = info["flops_per_point"]
-    for _ in range(args.warmup):
-        step()
-    torch.cuda.synchronize()
-    if dist:
-        dist.barrier()
-    l0 = sdag.launch_count()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with Clocks(local) as clk:
-        torch.cuda.synchronize()
-        e0.record(stream)
-        for _ in range(args.steps):
-            step()
-        e1.record(stream)
-        torch.cuda.synchronize()
-    launches = sdag.launch_count() - l0
-    ms = e0.elapsed_time(e1)
-    ms_t = torch.tensor([ms], dtype=torch.float64, device=red_dev)
-    pts_t = torch.tensor([float(pts_rank)], dtype=torch.float64, device=red_dev)
-    if dist:
-        dist.barrier()
-        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
-        dist.all_reduce(pts_t, op=dist.ReduceOp.SUM)
-    ms_max = float(ms_t.item())
-    total_pts = float(pts_t.item())
-    gflops = total_pts * flops_pt * args.steps / (ms_max * 1e-3) / 1e9
-
-    # dominant kernel: the sweep.  N=1: the step is exactly one launch.  N>1: time the
-    # local sweep kernel alone (same stream, same launch configuration).
-    kms = ms / max(1, launches) if not use_dist else None
-    if use_dist:
+            dd.apply([dB, dA], scalars=c, stream=stream, comm_stream=cs)
+        tdist.barrier()
+        ms, lps, clk = timed(step, args.steps, args.warmup, stream, local)
+        t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+        ms = float(t[0])
+        p = torch.tensor([float((part["k_hi"] - part["k_lo"]) * (ny - 8) * (nx - 8))], dtype=torch.float64,
+                         device="cuda")
+        tdist.all_reduce(p, op=tdist.ReduceOp.SUM)
+        pts_total = float(p[0])
+        # the dominant kernel alone (same stream, same launch configuration)
         ka, kb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        lp = dd.plan
         ka.record(stream)
         for _ in range(args.steps):
-            lp.apply(arrays, scalars=c, stream=stream)
+            kplan.apply([dB, dA], scalars=c, stream=stream)
         kb.record(stream)
         torch.cuda.synchronize()
         kms = ka.elapsed_time(kb) / args.steps
-    peak, peak_src = load_peaks()
-    bytes_launch = info["bytes_per_point"] * info["points"]
-    achieved = bytes_launch / (kms * 1e-3) / 1e9
-    traffic = load_traffic(info["variant"], ldims) if not use_dist else None
+    gflops = pts_total * info["flops_per_point"] / (ms * 1e-3) / 1e9
+    kernel = kplan.kernel_name(1)
+    counters = load_counters(info["variant"], (n, n, n)) if world == 1 else {}
+    roof = roofline(info if world == 1 else dict(info, points=(n - 8) ** 3), kms, 1, peak_hbm, peak_src, 0.0,
+                    counters, kernel)
 
+    # ---- e2e: the public call with host buffers, copies inside the timed region ----
     e2e = None
-    if not args.no_e2e and not use_dist:
-        hA = torch.from_numpy(A).pin_memory().numpy()
-        hB = torch.zeros(ldims, dtype=torch.float64).pin_memory().numpy()
-        ee = []
-        plan.apply_host([hB, hA], scalars=c, stream=stream)  # warm workspace
-        up = down = 0
-        for _ in range(max(3, min(args.steps, 5))):
-            t0 = time.perf_counter()
-            up, down = plan.apply_host([hB, hA], scalars=c, stream=stream)
-            ee.append(time.perf_counter() - t0)
-        t_e2e = statistics.median(ee)
-        e2e = {"value": info["points"] * flops_pt / t_e2e / 1e9, "unit": "GFLOP/s", "h2d_bytes_per_step": up,
-               "d2h_bytes_per_step": down, "ms_per_step": t_e2e * 1e3}
-    elif not args.no_e2e and use_dist:
-        # every rank: its slab (local layout, ghost planes included: the host holds
-        # them, so no exchange) host -> device from pinned memory, the sweep of its
-        # planes of the global interior, those planes device -> host, pipelined over
-        # z-chunks (sdag_dist_apply_host); wall time per step, max over ranks
-        hA = dA.cpu().pin_memory().numpy()
-        hB = torch.zeros((nza, ny, nx), dtype=torch.float64).pin_memory().numpy()
-        dd.apply_host([hB, hA], scalars=c, stream=stream)  # warm workspace
-        ee = []
-        up = down = 0
-        for it in range(max(3, min(args.steps, 5))):
-            if dist:
-                dist.barrier()
-            t0 = time.perf_counter()
-            up, down = dd.apply_host([hB, hA], scalars=c, stream=stream)
-            ee.append(time.perf_counter() - t0)
-        t_loc = torch.tensor([statistics.median(ee)], dtype=torch.float64, device=red_dev)
-        if dist:
-            dist.all_reduce(t_loc, op=dist.ReduceOp.MAX)
-        t_e2e = float(t_loc.item())
-        e2e = {"value": total_pts * flops_pt / t_e2e / 1e9, "unit": "GFLOP/s", "h2d_bytes_per_step": int(up),
-               "d2h_bytes_per_step": int(down), "ms_per_step": t_e2e * 1e3, "per_rank_bytes": True}
+    if not args.no_e2e:
+        if world == 1:
+            hA = dA.cpu().pin_memory().numpy()
+            hB = torch.zeros((n, n, n), dtype=torch.float64).pin_memory().numpy()
+            plan.apply_host([hB, hA], scalars=c, stream=stream)  # warm workspace
+            ee = []
+            for _ in range(max(3, min(args.steps, 5))):
+                t0 = time.perf_counter()
+                up, down = plan.apply_host([hB, hA], scalars=c, stream=stream)
+                ee.append(time.perf_counter() - t0)
+            te = statistics.median(ee)
+            e2e = {"value": info["points"] * info["flops_per_point"] / te / 1e9, "unit": "GFLOP/s",
+                   "h2d_bytes_per_step": int(up), "d2h_bytes_per_step": int(down), "ms_per_step": te * 1e3,
+                   "path": "sdag_apply_host (pipelined H2D / sweep / D2H over z-chunks)"}
+        else:
+            # owned planes host -> device (pinned), the NCCL-exchanged sweep, the
+            # computed planes device -> host; wall time per step, max over ranks
+            H = part["z0"] - g0
+            own = slice(H, H + part["nz_own"])
+            kk = slice(part["k_lo"], part["k_hi"])
+            hA = dA[own].cpu().pin_memory()
+            hB = torch.empty_like(dB[kk], device="cpu").pin_memory()
+            ee = []
+            for it in range(max(3, min(args.steps, 5)) + 1):
+                tdist.barrier()
+                t0 = time.perf_counter()
+                dA[own].copy_(hA, non_blocking=True)
+                dd.apply([dB, dA], scalars=c, stream=stream, comm_stream=cs)
+                hB.copy_(dB[kk], non_blocking=True)
+                stream.synchronize()
+                if it:
+                    ee.append(time.perf_counter() - t0)
+            t = torch.tensor([statistics.median(ee)], dtype=torch.float64, device="cuda")
+            tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+            te = float(t[0])
+            e2e = {"value": pts_total * info["flops_per_point"] / te / 1e9, "unit": "GFLOP/s",
+                   "h2d_bytes_per_step": int(hA.numel() * 8), "d2h_bytes_per_step": int(hB.numel() * 8),
+                   "ms_per_step": te * 1e3, "per_rank_bytes": True,
+                   "path": "owned planes H2D + Dist.apply (NCCL halo) + computed planes D2H"}
+    del dA, dB
+    torch.cuda.empty_cache()
 
+    # ---- per_config ----
+    per = {}
+    if not args.no_per_config:
+        if world == 1:
+            fp64 = sdag.fp64_peak()
+            for cid in [x for x in args.configs.split(",") if x]:
+                per[cid] = measure_config(cid, min(args.steps, 10), 3, peak_hbm, peak_src, fp64, tune=args.tune)
+            per["fp64_peak_tflops_measured"] = fp64 / 1e12
+        else:
+            per["5"] = measure_config5_slabs(tdist, rank, world, local, min(args.steps, 5), 3, comm, args.halo)
+
+    # ---- cpu_baseline (rank 0, N = 1): the oracle in a fresh process (no torch /
+    # CUDA threads competing with its OpenMP team: the same conditions as the
+    # reference arm) ----
     cpu = None
-    if rank == 0 and not use_dist and not args.no_cpu:
-        cpu = cpu_baseline_lap25(A, c)
+    if rank == 0 and world == 1 and not args.no_cpu:
+        r = subprocess.run([sys.executable, os.path.abspath(__file__), "--cpu-baseline-only",
+                            "--cpu-seconds", str(args.cpu_seconds)], capture_output=True, text=True, timeout=600)
+        cpu = json.loads(r.stdout.strip().splitlines()[-1]) if r.returncode == 0 and r.stdout.strip() else \
+            {"error": (r.stderr or "")[-300:]}
 
     if rank == 0:
-        line = {
-            "metric": METRIC, "value": gflops, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": CONFIGS[name][2], "stencil": name, "grid_per_gpu": list(ldims),
-                       "global_grid": list(gdims), "decomposition": f"z-slabs x{world}" if use_dist else "none",
-                       "halo": ("p2p" if p2p else "nccl") if use_dist else None,
-                       "variant": info["variant"], "flops_per_point": flops_pt,
-                       "bytes_per_point": info["bytes_per_point"],
-                       "l2": "input 1 GiB/GPU > 126 MB L2 (no flush needed)"},
-            "hbm_gbs": total_pts * info["bytes_per_point"] * args.steps / (ms_max * 1e-3) / 1e9,
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                         "kernel": "sdag_sweep<Lap25> " + info["variant"], "kernel_ms": kms},
-            "cpu_baseline": cpu,
-            "e2e": e2e,
-            "gpu_launches": launches,
-            "clocks": clk.summary(),
-        }
+        line = {"metric": METRIC, "value": gflops, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f64", "data": "synthetic (synth/ counter-based generator)",
+                "config": headline_config(world),
+                "plan": {"variant": info["variant"], "kernel": kernel, "flops_per_point": info["flops_per_point"],
+                         "bytes_per_point": info["bytes_per_point"], "tuned": bool(args.tune)},
+                "hbm_gbs": pts_total * info["bytes_per_point"] / (ms * 1e-3) / 1e9,
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(round(lps * args.steps)),
+                "clocks": clk, "per_config": per}
         print(json.dumps(line))
-    if dist:
-        dist.barrier()
-        dist.destroy_process_group()
+    if tdist:
+        tdist.barrier()
+        if comm:
+            sdag.nccl_comm_destroy(comm)
+        tdist.destroy_process_group()
     return 0
 
 

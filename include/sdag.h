@@ -133,10 +133,17 @@ sdag_status sdag_plan_create(const char *spec, const int64_t dims[3], const sdag
                              sdag_plan *out);
 sdag_status sdag_plan_info_get(sdag_plan plan, sdag_plan_info *out);
 /* kind: 0 = 3D array, 1 = 1D array, 2 = scalar; role (3D only): 0 in, 1 out, 2 inout.
- * For 1D arrays *role is the axis (0 = z, 1 = y, 2 = x).  Strings live as long as the plan. */
+ * For 1D arrays *role is the axis (0 = z, 1 = y, 2 = x) of the iterator indexing it,
+ * or -1 if the stencil never reads it (any length is accepted).  Strings live as long as the plan. */
 sdag_status sdag_plan_arg(sdag_plan plan, int32_t kind, int32_t idx, const char **name, int32_t *role);
 /* Candidate variants of this plan, 0 <= idx < info.n_variants. */
 sdag_status sdag_plan_variant_name(sdag_plan plan, int32_t idx, const char **name);
+/* The symbol of the kernel a sweep launches (demangled, as ncu lists it):
+ * sweeps = 1 -> the plan's single-sweep kernel (sdag_apply); sweeps = x > 1 ->
+ * the x-sweep temporally fused kernel sdag_apply_iterated uses (NEXT-1);
+ * INVALID_ARG if the plan has none.  Generated kernels read "nvrtc:<variant>".
+ * The string lives as long as the plan. */
+sdag_status sdag_plan_kernel_name(sdag_plan plan, int32_t sweeps, const char **name);
 /* Human-readable plan report (analysis counts, variant, launch geometry). */
 const char *sdag_plan_describe(sdag_plan plan);
 void sdag_plan_destroy(sdag_plan plan);
@@ -325,7 +332,8 @@ sdag_status sdag_dist_apply_iterated_loopback(sdag_dist *dists, int32_t nranks, 
  *   exchange handles: sdag_dist_p2p_handle(d, h) -> all-gather on the host ->
  *   sdag_dist_p2p_attach(d, 0, h_of(rank-1)), sdag_dist_p2p_attach(d, 1, h_of(rank+1))
  *   (or sdag_dist_p2p_attach_local(d, side, peer) for slabs of one process);
- *   fill buf0 (layout of sdag_dist_layout), then
+ *   fill the OWNED planes of buf0 (local planes [H, H + nz_own) of the layout of
+ *   sdag_dist_layout; ghost planes and buf1 need no filling), then
  *   sdag_dist_p2p_apply_iterated(d, T, scalars, n, stream)  -> result in buf[T&1].
  *
  * sdag_dist_p2p_alloc: the library allocates ONE device region holding buf0,
@@ -340,7 +348,11 @@ sdag_status sdag_dist_apply_iterated_loopback(sdag_dist *dists, int32_t nranks, 
  *   (its region is used directly; peer access is enabled if on another device).
  * sdag_dist_p2p_apply_iterated: T sweeps of a 1-in/1-out plan over buf0/buf1
  *   (fused launches as sdag_dist_apply_iterated), enqueued on `stream` only;
- *   bit-identical to the single-GPU schedule.  Consecutive calls on a rank are
+ *   bit-identical to the single-GPU schedule.  The FIRST call after
+ *   sdag_dist_p2p_alloc initialises buf1 from buf0 (owned planes locally, ghost
+ *   planes from the neighbours' bands), so the boundary ring (the x/y ring of
+ *   every plane, the global z-ring planes) is taken from buf0 at that call and
+ *   is never written afterwards.  Each call starts from buf0.  Consecutive calls on a rank are
  *   ordered against the neighbours' previous calls by the same flags.  A wait
  *   that does not complete within SDAG_P2P_TIMEOUT_S seconds (default 60)
  *   traps the kernel (the error surfaces at the next synchronisation). */

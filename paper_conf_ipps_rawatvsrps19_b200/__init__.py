@@ -58,6 +58,30 @@ def _ptr(t, what):
     return t.data_ptr()
 
 
+def _check_sizes(arrays3d, arrays1d, dims, axes, batch=1, device=None, host=False):
+    """The C ABI takes raw pointers, so an undersized buffer would be read or
+    written out of bounds on the device (TMA / stores) or on the host
+    (cudaMemcpy): check every 3D array holds batch*nz*ny*nx elements, every 1D
+    array the extent of its axis, and (device arrays) the plan's device."""
+    n = int(batch) * int(dims[0]) * int(dims[1]) * int(dims[2])
+    for q, t in enumerate(arrays3d):
+        cnt = int(t.size) if host else int(t.numel())
+        if cnt != n:
+            raise ValueError(f"grid array #{q} has {cnt} elements; the plan needs {n} "
+                             f"({'%d x ' % batch if batch > 1 else ''}{tuple(int(x) for x in dims)})")
+        if device is not None and not host and t.device.index != device:
+            raise ValueError(f"grid array #{q} is on {t.device}; the plan is on cuda:{device}")
+    if axes is not None:
+        for q, (t, ax) in enumerate(zip(arrays1d, axes)):
+            if ax < 0:  # never read by the stencil
+                continue
+            cnt = int(t.size) if host else int(t.numel())
+            if cnt != int(dims[ax]):
+                raise ValueError(f"1D array #{q} has {cnt} elements; its axis ({'zyx'[ax]}) has {int(dims[ax])}")
+            if device is not None and not host and t.device.index != device:
+                raise ValueError(f"1D array #{q} is on {t.device}; the plan is on cuda:{device}")
+
+
 def _arr(ptrs):
     return (ctypes.c_void_p * max(1, len(ptrs)))(*ptrs)
 
@@ -117,6 +141,7 @@ class Plan:
         o = _opts(order, device, tune, batch, variant, fusion)
         _check(self._L.sdag_plan_create(spec.encode(), d, ctypes.byref(o), ctypes.byref(self._h)))
         self._owned = True
+        self._device = int(o.device) if o.device >= 0 else None
 
     @classmethod
     def _borrow(cls, handle):
@@ -124,7 +149,21 @@ class Plan:
         p._L = _capi.lib()
         p._h = ctypes.c_void_p(handle)
         p._owned = False
+        p._device = None
         return p
+
+    def _meta(self):
+        """(dims, axis of each 1D formal), cached: plans are immutable"""
+        m = getattr(self, "_meta_cache", None)
+        if m is None:
+            dims = self.info["dims"]
+            axes = [a[3] for a in self.args() if a[0] == 1]
+            m = self._meta_cache = (dims, axes)
+        return m
+
+    def _sizes(self, arrays3d, arrays1d, batch=1, host=False):
+        dims, axes = self._meta()
+        _check_sizes(arrays3d, arrays1d, dims, axes, batch, getattr(self, "_device", None), host)
 
     def close(self):
         if getattr(self, "_owned", False) and self._h:
@@ -177,6 +216,12 @@ class Plan:
             out.append(nm.value.decode())
         return out
 
+    def kernel_name(self, sweeps: int = 1) -> str:
+        """symbol of the kernel a launch of `sweeps` fused sweeps runs (as ncu names it)"""
+        nm = ctypes.c_char_p()
+        _check(self._L.sdag_plan_kernel_name(self._h, int(sweeps), ctypes.byref(nm)))
+        return nm.value.decode()
+
     def describe(self) -> str:
         return self._L.sdag_plan_describe(self._h).decode()
 
@@ -200,12 +245,14 @@ class Plan:
 
     def apply(self, arrays3d, arrays1d=(), scalars=(), stream=None):
         p3 = [_ptr(t, "grid array") for t in arrays3d]
+        self._sizes(arrays3d, arrays1d)
         p1 = [_ptr(t, "1D array") for t in arrays1d]
         s, ns = _scal(scalars)
         _check(self._L.sdag_apply(self._h, _arr(p3), len(p3), _arr(p1), len(p1), s, ns, _stream_handle(stream)))
 
     def apply_batched(self, batch, arrays3d, arrays1d=(), scalars=(), stream=None):
         p3 = [_ptr(t, "grid array") for t in arrays3d]
+        self._sizes(arrays3d, arrays1d, batch=batch)
         p1 = [_ptr(t, "1D array") for t in arrays1d]
         s, ns = _scal(scalars)
         _check(self._L.sdag_apply_batched(self._h, int(batch), _arr(p3), len(p3), _arr(p1), len(p1), s, ns,
@@ -213,6 +260,8 @@ class Plan:
 
     def apply_iterated(self, buf0, buf1, T, scalars=(), stream=None):
         s, ns = _scal(scalars)
+        _ptr(buf0, "buf0"), _ptr(buf1, "buf1")
+        self._sizes([buf0, buf1], ())
         _check(self._L.sdag_apply_iterated(self._h, _ptr(buf0, "buf0"), _ptr(buf1, "buf1"), int(T), s, ns,
                                            _stream_handle(stream)))
 
@@ -223,6 +272,7 @@ class Plan:
         for a in list(host3d) + list(host1d):
             if not (isinstance(a, np.ndarray) and a.dtype == np.float64 and a.flags.c_contiguous):
                 raise TypeError("apply_host needs contiguous float64 numpy arrays")
+        self._sizes(host3d, host1d, host=True)
         p3 = [a.ctypes.data for a in host3d]
         p1 = [a.ctypes.data for a in host1d]
         s, ns = _scal(scalars)
@@ -366,6 +416,13 @@ class Dist:
         _check(self._L.sdag_dist_create(spec.encode(), d, ctypes.byref(o), int(rank), int(nranks),
                                         ctypes.c_void_p(comm or 0), ctypes.byref(self._h)))
         self.rank, self.nranks = rank, nranks
+        self._device = int(o.device) if o.device >= 0 else None
+
+    def _sizes(self, arrays3d, arrays1d, host=False):
+        """local layout (ghost planes included); 1D arrays sized to it too"""
+        dims = self.layout()[0]
+        axes = [a[3] for a in self.plan.args() if a[0] == 1]
+        _check_sizes(arrays3d, arrays1d, dims, axes, 1, self._device, host)
 
     def close(self):
         if self._h:
@@ -387,10 +444,15 @@ class Dist:
 
     @property
     def plan(self) -> Plan:
-        return Plan._borrow(self._L.sdag_dist_local_plan(self._h))
+        """Borrowed local plan (owned by this dist, which it keeps alive)."""
+        p = Plan._borrow(self._L.sdag_dist_local_plan(self._h))
+        p._dist = self
+        p._device = self._device
+        return p
 
     def apply(self, arrays3d, arrays1d=(), scalars=(), stream=None, comm_stream=None):
         p3 = [_ptr(t, "grid array") for t in arrays3d]
+        self._sizes(arrays3d, arrays1d)
         p1 = [_ptr(t, "1D array") for t in arrays1d]
         s, ns = _scal(scalars)
         cs = ctypes.c_void_p(0) if comm_stream is None else _stream_handle(comm_stream)
@@ -399,12 +461,19 @@ class Dist:
 
     def apply_iterated(self, buf0, buf1, T, scalars=(), stream=None, comm_stream=None):
         s, ns = _scal(scalars)
+        _ptr(buf0, "buf0"), _ptr(buf1, "buf1")
+        self._sizes([buf0, buf1], ())
         cs = ctypes.c_void_p(0) if comm_stream is None else _stream_handle(comm_stream)
         _check(self._L.sdag_dist_apply_iterated(self._h, _ptr(buf0, "buf0"), _ptr(buf1, "buf1"), int(T), s, ns,
                                                 _stream_handle(stream), cs))
 
     @staticmethod
     def apply_iterated_loopback(dists, bufs0, bufs1, T, scalars=(), stream=None):
+        if not (len(dists) == len(bufs0) == len(bufs1)):
+            raise ValueError("one buf0 and one buf1 per dist")
+        for d, x, y in zip(dists, bufs0, bufs1):
+            _ptr(x, "buf0"), _ptr(y, "buf1")
+            d._sizes([x, y], ())
         hs = (ctypes.c_void_p * len(dists))(*[d._h.value for d in dists])
         b0 = _arr([_ptr(t, "buf0") for t in bufs0])
         b1 = _arr([_ptr(t, "buf1") for t in bufs1])
@@ -420,6 +489,7 @@ class Dist:
         for a in list(host3d) + list(host1d):
             if not (isinstance(a, np.ndarray) and a.dtype == np.float64 and a.flags.c_contiguous):
                 raise TypeError("apply_host needs contiguous float64 numpy arrays")
+        self._sizes(host3d, host1d, host=True)
         p3 = [a.ctypes.data for a in host3d]
         p1 = [a.ctypes.data for a in host1d]
         s, ns = _scal(scalars)
@@ -431,13 +501,15 @@ class Dist:
     # ---- peer-memory halo path (NVLink P2P stores from the sweep kernels) ----
     def p2p_alloc(self):
         """(buf0, buf1): the library-owned slab buffers of sdag_dist_p2p_alloc as
-        float64 CUDA tensors of the local layout (views; valid while this dist lives)"""
+        float64 CUDA tensors of the local layout (zero-copy views that keep this
+        dist -- the owner of the memory -- alive).  Fill buf0's owned planes; the
+        first p2p_apply_iterated initialises buf1 and the ghost planes."""
         import torch
         b0, b1 = ctypes.c_void_p(), ctypes.c_void_p()
         _check(self._L.sdag_dist_p2p_alloc(self._h, ctypes.byref(b0), ctypes.byref(b1)))
         shape = tuple(int(x) for x in self.layout()[0])
-        dev = torch.device("cuda", torch.cuda.current_device())
-        return tuple(torch.as_tensor(_DeviceView(b.value, shape), device=dev) for b in (b0, b1))
+        dev = torch.device("cuda", self._device if self._device is not None else torch.cuda.current_device())
+        return tuple(torch.as_tensor(_DeviceView(b.value, shape, owner=self), device=dev) for b in (b0, b1))
 
     def p2p_handle(self) -> bytes:
         h = ctypes.create_string_buffer(64)
@@ -463,7 +535,8 @@ class Dist:
 class _DeviceView:
     """__cuda_array_interface__ of a float64 C-order device buffer (zero copy)"""
 
-    def __init__(self, ptr, shape):
+    def __init__(self, ptr, shape, owner=None):
+        self._owner = owner  # torch.as_tensor keeps this object (and so the owner) alive
         self.__cuda_array_interface__ = {"shape": shape, "typestr": "<f8", "data": (int(ptr), False),
                                          "version": 3, "strides": None}
 

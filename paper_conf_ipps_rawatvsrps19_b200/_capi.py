@@ -54,6 +54,7 @@ def lib():
             "sdag_plan_arg": (S, [P, c_i32, c_i32, ctypes.POINTER(c_char_p), ctypes.POINTER(c_i32)]),
             "sdag_plan_variant_name": (S, [P, c_i32, ctypes.POINTER(c_char_p)]),
             "sdag_plan_describe": (c_char_p, [P]),
+            "sdag_plan_kernel_name": (S, [P, c_i32, ctypes.POINTER(c_char_p)]),
             "sdag_plan_destroy": (None, [P]),
             "sdag_apply": (S, [P, ctypes.POINTER(c_void_p), c_i32, ctypes.POINTER(c_void_p), c_i32, c_dblp, c_i32,
                                P]),
@@ -129,7 +130,7 @@ class Profile(ctypes.Structure):
 
 # every symbol include/sdag.h declares (checked by tests/test_capi_symbols.py)
 EXPORTED = [
-    "sdag_plan_opts_init", "sdag_plan_create", "sdag_plan_info_get", "sdag_plan_arg", "sdag_plan_variant_name",
+    "sdag_plan_opts_init", "sdag_plan_create", "sdag_plan_info_get", "sdag_plan_arg", "sdag_plan_variant_name", "sdag_plan_kernel_name",
     "sdag_plan_describe", "sdag_plan_destroy", "sdag_apply", "sdag_apply_batched", "sdag_apply_iterated",
     "sdag_program_create", "sdag_program_info", "sdag_program_arg", "sdag_program_stage", "sdag_program_apply",
     "sdag_program_destroy",

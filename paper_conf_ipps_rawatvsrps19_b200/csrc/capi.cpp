@@ -2,6 +2,9 @@
 // exception -> sdag_status translation, thread-local error text.
 #include <cuda_runtime.h>
 
+#include <cxxabi.h>
+
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -79,7 +82,9 @@ sdag_status sdag_plan_arg(sdag_plan plan, int32_t kind, int32_t idx, const char 
         if (idx < 0 || idx >= p->st.n_of(k)) throw sdag::Error(SDAG_ERR_INVALID_ARG, "index out of range");
         const sdag::Formal &f = p->st.formal(k, idx);
         if (name) *name = f.name.c_str();
-        if (role) *role = (k == sdag::ArgKind::Array3D) ? int32_t(f.role) : (k == sdag::ArgKind::Array1D ? f.axis : -1);
+        if (role)
+            *role = (k == sdag::ArgKind::Array3D) ? int32_t(f.role)
+                    : (k == sdag::ArgKind::Array1D ? (f.role == sdag::Role::Unused ? -1 : f.axis) : -1);
     });
 }
 
@@ -88,6 +93,39 @@ sdag_status sdag_plan_variant_name(sdag_plan plan, int32_t idx, const char **nam
         sdag::Plan *p = P(plan);
         if (idx < 0 || idx >= int(p->cands.size())) throw sdag::Error(SDAG_ERR_INVALID_ARG, "index out of range");
         if (name) *name = p->cands[idx]->variant.c_str();
+    });
+}
+
+sdag_status sdag_plan_kernel_name(sdag_plan plan, int32_t sweeps, const char **name) {
+    return guard([&] {
+        sdag::Plan *p = P(plan);
+        if (!name) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null name");
+        const sdag::KernelDesc *k = nullptr;
+        if (sweeps == 1) {
+            k = &p->kernel();
+        } else {
+            for (const sdag::KernelDesc *f : p->fused)
+                if (f->tsteps == sweeps) {
+                    k = f;
+                    break;
+                }
+        }
+        if (!k) throw sdag::Error(SDAG_ERR_INVALID_ARG, "the plan has no " + std::to_string(sweeps) + "-sweep kernel");
+        std::lock_guard<std::mutex> lk(p->mu);
+        auto it = p->kname.find(sweeps);
+        if (it == p->kname.end()) {
+            std::string s = "nvrtc:" + k->variant;  // generated (NEXT-4) kernels
+            const char *mangled = nullptr;
+            if (k->fn && cudaFuncGetName(&mangled, k->fn) == cudaSuccess && mangled) {
+                int st = 0;
+                char *dm = abi::__cxa_demangle(mangled, nullptr, nullptr, &st);
+                s = (st == 0 && dm) ? dm : mangled;
+                std::free(dm);
+            }
+            cudaGetLastError();
+            it = p->kname.emplace(sweeps, s).first;
+        }
+        *name = it->second.c_str();
     });
 }
 

@@ -88,6 +88,7 @@ struct NcclApi {
     ncclResult_t (*Recv)(void *, size_t, int, int, ncclComm_t, cudaStream_t) = nullptr;
     ncclResult_t (*GroupStart)() = nullptr;
     ncclResult_t (*GroupEnd)() = nullptr;
+    ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t *) = nullptr;
     const char *(*GetErrorString)(ncclResult_t) = nullptr;
     std::string err;
 };
@@ -112,6 +113,7 @@ const NcclApi &nccl() {
         x.GroupStart = reinterpret_cast<decltype(x.GroupStart)>(sym("ncclGroupStart"));
         x.GroupEnd = reinterpret_cast<decltype(x.GroupEnd)>(sym("ncclGroupEnd"));
         x.GetErrorString = reinterpret_cast<decltype(x.GetErrorString)>(sym("ncclGetErrorString"));
+        x.CommGetAsyncError = reinterpret_cast<decltype(x.CommGetAsyncError)>(sym("ncclCommGetAsyncError"));
         if (!x.GetUniqueId || !x.CommInitRank || !x.Send || !x.Recv || !x.GroupStart || !x.GroupEnd)
             x.err = "libnccl.so.2 lacks the point-to-point API";
         return x;
@@ -138,9 +140,13 @@ void nccl_unique_id(uint8_t id[128]) {
 void *nccl_comm_create(const uint8_t id[128], int nranks, int rank, int device) {
     ncclUniqueId u;
     std::memcpy(u.internal, id, 128);
+    int prev = -1;
+    check_cuda(cudaGetDevice(&prev), "cudaGetDevice");
     if (device >= 0) check_cuda(cudaSetDevice(device), "cudaSetDevice");
     ncclComm_t c = nullptr;
-    nck(nccl().CommInitRank(&c, nranks, u, rank), "ncclCommInitRank");
+    const ncclResult_t r = nccl().CommInitRank(&c, nranks, u, rank);
+    if (prev >= 0) cudaSetDevice(prev);  // the caller's current device is left as it was
+    nck(r, "ncclCommInitRank");
     return c;
 }
 
@@ -250,19 +256,40 @@ void exchange_nccl(Dist *d, double *const *a3, cudaStream_t comm, int planes) {
     const size_t cnt = plane * size_t(planes);
     const Halo h = halo_schedule(d->slab, planes);
     auto c = static_cast<ncclComm_t>(d->comm);
+    // every call between GroupStart and GroupEnd is made even after a failure,
+    // and GroupEnd always runs: an open group would corrupt every later call on
+    // the communicator.  The first error is reported after the group is closed.
+    ncclResult_t first = 0;
+    const char *first_what = nullptr;
+    auto call = [&](ncclResult_t r, const char *what) {
+        if (r != 0 && first == 0) {
+            first = r;
+            first_what = what;
+        }
+    };
     nck(N.GroupStart(), "ncclGroupStart");
     for (int f : halo_arrays(d)) {
         double *a = a3[f];
         if (h.lo_send >= 0) {
-            nck(N.Send(a + size_t(h.lo_send) * plane, cnt, ncclFloat64, d->rank - 1, c, comm), "ncclSend");
-            nck(N.Recv(a + size_t(h.lo_recv) * plane, cnt, ncclFloat64, d->rank - 1, c, comm), "ncclRecv");
+            call(N.Send(a + size_t(h.lo_send) * plane, cnt, ncclFloat64, d->rank - 1, c, comm), "ncclSend");
+            call(N.Recv(a + size_t(h.lo_recv) * plane, cnt, ncclFloat64, d->rank - 1, c, comm), "ncclRecv");
         }
         if (h.up_send >= 0) {
-            nck(N.Send(a + size_t(h.up_send) * plane, cnt, ncclFloat64, d->rank + 1, c, comm), "ncclSend");
-            nck(N.Recv(a + size_t(h.up_recv) * plane, cnt, ncclFloat64, d->rank + 1, c, comm), "ncclRecv");
+            call(N.Send(a + size_t(h.up_send) * plane, cnt, ncclFloat64, d->rank + 1, c, comm), "ncclSend");
+            call(N.Recv(a + size_t(h.up_recv) * plane, cnt, ncclFloat64, d->rank + 1, c, comm), "ncclRecv");
         }
     }
-    nck(N.GroupEnd(), "ncclGroupEnd");
+    const ncclResult_t ge = N.GroupEnd();
+    if (first != 0) nck(first, first_what);
+    nck(ge, "ncclGroupEnd");
+    // SDAG_NCCL_CHECK=1 (debug): poll the communicator's asynchronous error
+    // after every exchange (failure detection)
+    static const bool async_check = std::getenv("SDAG_NCCL_CHECK") && std::getenv("SDAG_NCCL_CHECK")[0] == '1';
+    if (async_check && N.CommGetAsyncError) {
+        ncclResult_t ae = 0;
+        nck(N.CommGetAsyncError(c, &ae), "ncclCommGetAsyncError");
+        nck(ae, "NCCL asynchronous error");
+    }
 }
 
 // local planes of the global z-interior (multi-sweep kernels keep the rest fixed)
@@ -343,13 +370,12 @@ void dist_apply(Dist *d, double *const *a3, int n3, const double *const *a1, int
     if (!d) throw Error(SDAG_ERR_INVALID_ARG, "null dist");
     Plan *p = d->local;
     if (p->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
-    if (n3 != p->n3() || n1 != p->n1() || ns != p->ns()) throw Error(SDAG_ERR_INVALID_ARG, "argument counts");
-    for (int f = 0; f < n3; f++)
-        if (!a3[f]) throw Error(SDAG_ERR_INVALID_ARG, "null grid array");
+    // counts, null pointers, null scalars, output aliasing: nothing enqueued on a bad call
+    plan_validate(p, a3, n3, a1, n1, s, ns, 1);
     if (p->kernel().tma)
         for (int f = 0; f < n3; f++)
             if (reinterpret_cast<uintptr_t>(a3[f]) % 16) throw Error(SDAG_ERR_INVALID_ARG, "grid arrays must be 16-B aligned");
-    check_cuda(cudaSetDevice(p->device), "cudaSetDevice");  // libsdag's runtime: bind the plan's device
+    DeviceGuard dg(p);  // libsdag's runtime: bind the plan's device, restore the caller's
     sweep_split(d, p->kernel(), a3, a1, s, compute, comm_stream(d, comm), true);
 }
 
@@ -360,10 +386,10 @@ void dist_apply_iterated(Dist *d, double *b0, double *b1, int T, const double *s
     if (p->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
     if (p->n3() != 2 || p->an.n_in != 1 || p->an.n_out != 1 || p->n1() != 0)
         throw Error(SDAG_ERR_INVALID_ARG, "iterated dist apply needs a 1-input 1-output plan");
-    if (ns != p->ns() || !b0 || !b1 || b0 == b1 || T < 0) throw Error(SDAG_ERR_INVALID_ARG, "bad arguments");
+    if (ns != p->ns() || (ns > 0 && !s) || !b0 || !b1 || b0 == b1 || T < 0) throw Error(SDAG_ERR_INVALID_ARG, "bad arguments");
     int fin = -1, fout = -1;
     for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
-    check_cuda(cudaSetDevice(p->device), "cudaSetDevice");
+    DeviceGuard dg(p);
     cudaStream_t cs = comm_stream(d, comm);
     double *bufs[2] = {b0, b1};
     int cur = 0;
@@ -385,11 +411,11 @@ void dist_apply_iterated_loopback(Dist **ds, int n, double *const *b0, double *c
         if (ds[r]->time_tile != ds[0]->time_tile) throw Error(SDAG_ERR_INVALID_ARG, "dists must share time_tile");
     }
     Plan *p0 = ds[0]->local;
-    if (p0->n3() != 2 || p0->an.n_in != 1 || p0->an.n_out != 1 || p0->n1() != 0 || ns != p0->ns() || T < 0)
+    if (p0->n3() != 2 || p0->an.n_in != 1 || p0->an.n_out != 1 || p0->n1() != 0 || ns != p0->ns() || (ns > 0 && !s) || T < 0)
         throw Error(SDAG_ERR_INVALID_ARG, "iterated loopback needs a 1-input 1-output plan");
     int fin = -1, fout = -1;
     for (int f = 0; f < 2; f++) (p0->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
-    check_cuda(cudaSetDevice(p0->device), "cudaSetDevice");
+    DeviceGuard dg(p0);
     const int64_t rz = ds[0]->rz;
     const size_t plane = size_t(p0->dims[1] * p0->dims[2]);
     // every rank follows rank 0's schedule (same plan, same buffers' alignment class)
@@ -484,7 +510,7 @@ void dist_apply_host(Dist *d, double *const *h3, int n3, const double *const *h1
 void dist_p2p_alloc(Dist *d, double **buf0, double **buf1) {
     if (!d) throw Error(SDAG_ERR_INVALID_ARG, "null dist");
     if (d->local->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
-    check_cuda(cudaSetDevice(d->local->device), "cudaSetDevice");
+    DeviceGuard dg(d->local);
     if (!d->p2p_base) {
         const int64_t *dims = d->local->dims;
         d->p2p_buf_bytes = p2p_buf_bytes(dims[0], dims[1], dims[2]);
@@ -497,6 +523,7 @@ void dist_p2p_alloc(Dist *d, double **buf0, double **buf1) {
         check_cuda(cudaMemset(d->p2p_base, 0, total), "cudaMemset(p2p)");
         check_cuda(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
         d->epoch = 0;
+        d->p2p_synced = false;
     }
     if (buf0) *buf0 = d->p2p_buf[0];
     if (buf1) *buf1 = d->p2p_buf[1];
@@ -513,7 +540,7 @@ void dist_p2p_handle(Dist *d, uint8_t handle[64]) {
 void dist_p2p_attach(Dist *d, int side, const uint8_t handle[64]) {
     if (!d || !d->p2p_base) throw Error(SDAG_ERR_INVALID_ARG, "call sdag_dist_p2p_alloc first");
     if (side != 0 && side != 1) throw Error(SDAG_ERR_INVALID_ARG, "side must be 0 (lower) or 1 (upper)");
-    check_cuda(cudaSetDevice(d->local->device), "cudaSetDevice");
+    DeviceGuard dg(d->local);
     cudaIpcMemHandle_t h;
     std::memcpy(&h, handle, 64);
     void *m = nullptr;
@@ -532,7 +559,7 @@ void dist_p2p_attach_local(Dist *d, int side, Dist *peer) {
         int ok = 0;
         check_cuda(cudaDeviceCanAccessPeer(&ok, d->local->device, peer->local->device), "cudaDeviceCanAccessPeer");
         if (!ok) throw Error(SDAG_ERR_DEVICE, "devices cannot access each other's memory");
-        check_cuda(cudaSetDevice(d->local->device), "cudaSetDevice");
+        DeviceGuard dg(d->local);
         const cudaError_t e = cudaDeviceEnablePeerAccess(peer->local->device, 0);
         if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) check_cuda(e, "cudaDeviceEnablePeerAccess");
         cudaGetLastError();
@@ -545,7 +572,7 @@ void dist_p2p_apply_iterated(Dist *d, int T, const double *s, int ns, cudaStream
     Plan *p = d->local;
     if (p->n3() != 2 || p->an.n_in != 1 || p->an.n_out != 1 || p->n1() != 0)
         throw Error(SDAG_ERR_INVALID_ARG, "iterated dist apply needs a 1-input 1-output plan");
-    if (ns != p->ns() || T < 0) throw Error(SDAG_ERR_INVALID_ARG, "bad arguments");
+    if (ns != p->ns() || (ns > 0 && !s) || T < 0) throw Error(SDAG_ERR_INVALID_ARG, "bad arguments");
     const Slab &S = d->slab;
     const int has[2] = {S.has_lower, S.has_upper};
     for (int q = 0; q < 2; q++)
@@ -554,7 +581,7 @@ void dist_p2p_apply_iterated(Dist *d, int T, const double *s, int ns, cudaStream
                                                   " neighbour attached (sdag_dist_p2p_attach)");
     int fin = -1, fout = -1;
     for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
-    check_cuda(cudaSetDevice(p->device), "cudaSetDevice");
+    DeviceGuard dg(p);
     if (T == 0) return;
 
     const int64_t H = S.halo;
@@ -563,13 +590,14 @@ void dist_p2p_apply_iterated(Dist *d, int T, const double *s, int ns, cudaStream
     double **buf = d->p2p_buf;
     // bands, in my local planes: [H, 2H) goes to the lower neighbour, [nz_own, nz_own+H) to the upper
     const int64_t band_lo[2] = {H, S.nz_own};
-    auto push = [&](int b) {  // my bands of buffer b -> the neighbours' ghost planes of their buffer b
+    auto push_to = [&](int b, int pb) {  // my bands of buffer b -> the neighbours' ghost planes of their buffer pb
         for (int q = 0; q < 2; q++)
             if (has[q])
-                check_cuda(cudaMemcpyAsync(d->peer_buf[q][b] + size_t(band_lo[q] + d->peer_shift[q]) * plane,
+                check_cuda(cudaMemcpyAsync(d->peer_buf[q][pb] + size_t(band_lo[q] + d->peer_shift[q]) * plane,
                                            buf[b] + size_t(band_lo[q]) * plane, band, cudaMemcpyDefault, st),
                            "p2p band push");
     };
+    auto push = [&](int b) { push_to(b, b); };
     auto signal = [&](uint32_t v) {
         p2p_signal(has[0] ? d->peer_flag[0] : nullptr, has[1] ? d->peer_flag[1] : nullptr, v, st);
         d->epoch = v;
@@ -591,6 +619,20 @@ void dist_p2p_apply_iterated(Dist *d, int T, const double *s, int ns, cudaStream
     }
 
     wait(d->epoch);  // the neighbours' previous call is over (first call: 0)
+    if (!d->p2p_synced) {
+        // First call after sdag_dist_p2p_alloc: the caller filled buf0's owned
+        // planes.  buf1's owned planes get buf0's (its x/y ring and the global
+        // z-ring planes are never written by a sweep), and my bands of buf0
+        // go into the neighbours' buf1 ghost planes too (their x/y ring is
+        // never written by the neighbours' mirrored stores, which cover the
+        // interior only).  All of it precedes signal(base), which gates every
+        // neighbour access to those planes, and nobody else writes my owned
+        // planes: race-free.
+        check_cuda(cudaMemcpyAsync(buf[1] + size_t(H) * plane, buf[0] + size_t(H) * plane,
+                                   size_t(S.nz_own) * plane * 8, cudaMemcpyDeviceToDevice, st), "p2p buf1 init");
+        push_to(0, 1);
+        d->p2p_synced = true;
+    }
     push(0);
     const uint32_t base = d->epoch + 1;
     signal(base);

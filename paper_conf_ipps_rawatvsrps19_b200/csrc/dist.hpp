@@ -52,6 +52,7 @@ struct Dist {
     int64_t peer_shift[2] = {0, 0};       // my local plane k is the neighbour's plane k + shift
     void *peer_ipc[2] = {};               // opened IPC mappings (closed in ~Dist)
     uint32_t epoch = 0;                   // last flag value this rank signalled
+    bool p2p_synced = false;              // buf1 initialised from buf0 (first p2p call)
     ~Dist();
 };
 

@@ -74,6 +74,7 @@ struct Plan {
     std::mutex host_mu;              // sdag_apply_host calls on one plan are serialised (shared workspace)
     cudaStream_t hs_up = nullptr;    // sdag_apply_host copy streams (H2D, D2H), created on first use
     cudaStream_t hs_down = nullptr;
+    std::map<int, std::string> kname;  // sdag_plan_kernel_name results (guarded by mu)
 
     ~Plan();
     const KernelDesc &kernel() const { return *cands[chosen]; }
@@ -142,6 +143,19 @@ void apply_host(Plan *p, double *const *h3, int n3, const double *const *h1, int
                 cudaStream_t stream, int64_t *h2d, int64_t *d2h,
                 const int64_t *krange = nullptr);
 void check_cuda(cudaError_t e, const char *what);
+// binds the plan's device for the duration of an entry point and restores the
+// caller's current device on exit (also on a throw)
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(const Plan *p) {
+        if (p->host_only) throw Error(SDAG_ERR_DEVICE, "plan was created host-only (SDAG_DEVICE_NONE)");
+        check_cuda(cudaGetDevice(&prev), "cudaGetDevice");
+        if (prev != p->device) check_cuda(cudaSetDevice(p->device), "cudaSetDevice");
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
 // jit.cu (NEXT-4)
 std::string jit_body_source(const Plan &p, const std::string &sname, int rzr);
 void jit_build_candidates(Plan *p);

@@ -358,18 +358,6 @@ static void validate_arrays(Plan *p, double *const *a3, int n3, const double *co
     }
 }
 
-struct DeviceGuard {
-    int prev = -1;
-    explicit DeviceGuard(const Plan *p) {
-        if (p->host_only) throw Error(SDAG_ERR_DEVICE, "plan was created host-only (SDAG_DEVICE_NONE)");
-        check_cuda(cudaGetDevice(&prev), "cudaGetDevice");
-        if (prev != p->device) check_cuda(cudaSetDevice(p->device), "cudaSetDevice");
-    }
-    ~DeviceGuard() {
-        if (prev >= 0) cudaSetDevice(prev);
-    }
-};
-
 void plan_validate(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns,
                    int batch) {
     if (batch < 1) throw Error(SDAG_ERR_INVALID_ARG, "batch must be >= 1");

@@ -624,6 +624,7 @@ struct Resolver {
         if (fo.axis >= 0 && fo.axis != ax)
             fail(SDAG_ERR_UNSUPPORTED, ix.line, ix.col, "1D array '" + r.s + "' indexed by two iterators");
         fo.axis = ax;
+        fo.role = Role::In;  // a read 1D array (unread ones stay Unused)
         n.kind = Node::Load1;
         n.ref = fo.kind_index;
         n.off[0] = ix.off;

@@ -166,3 +166,29 @@ def rhs4_inputs(dims, cfg="cfg4"):
     }
     scal = {"tf": 0.75, "i6": 1.0 / 6.0, "i144": 1.0 / 144.0, "cof": 1.0, "a1": 1.0}
     return ins, scal
+
+
+# ---------------------------------------------------------------------------
+# The same recipes as data (bench.py builds the BASELINE-size inputs on the
+# device from these with uniform_torch -- bit-identical to the *_inputs()
+# arrays of the same cfg key, checked by tests/test_synth.py).
+# recipe(name) -> (cfg key, {3D array: (lo, hi)}, {1D array: (lo, hi)}, scalars)
+# ---------------------------------------------------------------------------
+
+_RECIPES = {
+    "jacobi7": ("cfg1", {"A": (-1.0, 1.0)}, {}, {"a": 0.5, "b": 0.25, "h2inv": 4.0}),
+    "lap25": ("cfg2", {"A": (-1.0, 1.0)}, {}, LAP25_COEFS),
+    "smooth27": ("cfg5", {"A": (-1.0, 1.0)}, {}, SMOOTH27_W),
+    "hypterm": ("cfg3", {"cons_1": (0.5, 1.5), "cons_2": (0.5, 1.5), "cons_3": (0.5, 1.5), "cons_4": (0.5, 1.5),
+                         "q_1": (-1.0, 1.0), "q_2": (-1.0, 1.0), "q_3": (-1.0, 1.0), "q_4": (0.5, 1.5)}, {},
+                {"dxinv0": 0.5, "dxinv1": 0.25, "dxinv2": 0.125, **HYPTERM_C}),
+    "rhs4center": ("cfg4", {"u0": (-1.0, 1.0), "u1": (-1.0, 1.0), "u2": (-1.0, 1.0), "mu": (1.0, 2.0),
+                            "la": (1.0, 2.0), "uacc0": (-1.0, 1.0), "uacc1": (-1.0, 1.0), "uacc2": (-1.0, 1.0)},
+                   {"strx": (0.5, 1.5), "stry": (0.5, 1.5), "strz": (0.5, 1.5)},
+                   {"tf": 0.75, "i6": 1.0 / 6.0, "i144": 1.0 / 144.0, "cof": 1.0, "a1": 1.0}),
+}
+
+
+def recipe(name):
+    cfg, a3, a1, sc = _RECIPES[name]
+    return cfg, dict(a3), dict(a1), dict(sc)

@@ -5,6 +5,8 @@ reading R13:  e_p = |g_p - o_p| / max(|o_p|, A_p) <= TOL, A_p the abs-mode
 oracle value."""
 from __future__ import annotations
 
+import os
+
 import numpy as np
 
 import oracle
@@ -31,6 +33,36 @@ def scaled_err(g, o, a):
     with np.errstate(invalid="ignore", divide="ignore"):
         e = np.where(den > 0, np.abs(g - o) / np.where(den > 0, den, 1.0), np.abs(g - o))
     return float(np.max(e)) if e.size else 0.0
+
+
+# worst scaled error e_p seen per test (and per output): printed at the end of
+# the session by tests/conftest.py and written to $SDAG_PARITY_LOG (JSON) so
+# the margin under the 1e-12 gate is visible, not just pass/fail.
+WORST: dict = {}
+
+
+def _test_id():
+    return os.environ.get("PYTEST_CURRENT_TEST", "?").split(" ")[0]
+
+
+def gate(g, o, a, what=""):
+    """The north-star gate (BASELINE.json, DESIGN R13):
+    e_p = |g_p - o_p| / max(|o_p|, A_p) <= 1e-12 at every compared point, A_p
+    the abs-mode value (for iterates and programs: the abs-mode iterate /
+    composition -- the gate itself is never widened).  Records the worst e_p,
+    the normwise error max|g-o|/max|o| and the number of points compared."""
+    g, o, a = np.asarray(g, dtype=np.float64), np.asarray(o, dtype=np.float64), np.asarray(a, dtype=np.float64)
+    e = scaled_err(g, o, a)
+    mo = float(np.max(np.abs(o))) if o.size else 0.0
+    nw = float(np.max(np.abs(g - o))) / mo if mo > 0 else 0.0
+    key = _test_id() + (f" [{what}]" if what else "")
+    prev = WORST.get(key)
+    if prev is None or e > prev["e_p"]:
+        WORST[key] = {"e_p": e, "normwise": nw, "points": int(o.size) + (prev["points"] if prev else 0)}
+    else:
+        prev["points"] += int(o.size)
+    assert e <= TOL, f"{key}: scaled error {e:.3e} > {TOL:.0e}"
+    return e
 
 
 def make_case(name, dims, cfg="t"):
@@ -97,9 +129,7 @@ def check(name, dims, g, case):
     I = interior(dims, R)
     worst = 0.0
     for m, (gm, om, am) in enumerate(zip(g, case["o"], case["a"])):
-        e = scaled_err(gm[I], om[I], am[I])
-        worst = max(worst, e)
-        assert e <= TOL, f"{name} output {m}: scaled error {e:.3e} > {TOL}"
+        worst = max(worst, gate(gm[I], om[I], am[I], what=f"{name} output {m}"))
         ring = ring_mask(dims, R)
         if case["inout"]:
             assert np.array_equal(gm[ring], case["inout"][m][ring]), f"{name} output {m}: ring modified"

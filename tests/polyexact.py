@@ -98,6 +98,47 @@ class Poly:
         return out.reshape(shape)
 
 
+    def grid_fast(self, shape, origin):
+        """Same values as grid() for large grids: every coefficient must be a
+        dyadic rational (denominator 2^e); D*p is evaluated in int64 numpy and
+        divided by D = 2^e in float64 (exact).  The a-priori bound
+        sum |D c| max|x|^a max|y|^b max|z|^c < 2^53 is asserted first, so no
+        partial sum can overflow int64 or lose a bit in the final float."""
+        D = 1
+        for v in self.c.values():
+            d = Fraction(v).denominator
+            assert d & (d - 1) == 0, f"coefficient {v} is not dyadic"
+            D = max(D, d)
+        nz, ny, nx = shape
+        oz, oy, ox = origin
+        mx = max(abs(0 - ox), abs(nx - 1 - ox))
+        my = max(abs(0 - oy), abs(ny - 1 - oy))
+        mz = max(abs(0 - oz), abs(nz - 1 - oz))
+        bound = sum(abs(int(Fraction(v) * D)) * mx ** a * my ** b * mz ** c for (a, b, c), v in self.c.items())
+        assert bound < 2 ** 53, f"grid values may reach {bound} >= 2^53"
+        x = np.arange(nx, dtype=np.int64) - ox
+        y = np.arange(ny, dtype=np.int64) - oy
+        z = np.arange(nz, dtype=np.int64) - oz
+        acc = np.zeros(shape, dtype=np.int64)
+        for (a, b, c), v in self.c.items():
+            cv = int(Fraction(v) * D)
+            yz = (cv * z[:, None] ** c) * (y[None, :] ** b)  # [nz][ny]
+            acc += yz[:, :, None] * (x ** a)[None, None, :]
+        out = acc.astype(np.float64)
+        if D != 1:
+            out /= float(D)
+        return out
+
+    def bound(self, shape, origin):
+        """max over the grid of sum |c| |x|^a |y|^b |z|^c (exact, Fraction)."""
+        nz, ny, nx = shape
+        oz, oy, ox = origin
+        mx = max(ox, nx - 1 - ox)
+        my = max(oy, ny - 1 - oy)
+        mz = max(oz, nz - 1 - oz)
+        return sum(abs(Fraction(v)) * mx ** a * my ** b * mz ** c for (a, b, c), v in self.c.items())
+
+
 def random_poly(rng: random.Random, max_deg_axis=(3, 3, 3), max_total=None, coef=3, nterms=8) -> Poly:
     terms = {}
     for _ in range(nterms):

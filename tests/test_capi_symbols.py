@@ -76,3 +76,20 @@ def test_plain_c_client(tmp_path):
     assert "array B role 1" in out.stdout and "array A role 0" in out.stdout
     assert "bad spec -> status 2 (PARSE)" in out.stdout
     assert "trivial fission: 3 stencils" in out.stdout
+
+
+def test_binding_rejects_undersized_host_buffers():
+    """the binding checks element counts before handing raw pointers
+    to the C ABI (an undersized buffer would be read/written out of bounds)."""
+    import numpy as np
+    import pytest as _pt
+
+    import paper_conf_ipps_rawatvsrps19_b200 as sdag
+    plan = sdag.Plan(sdag.spec_text("jacobi7"), (8, 9, 10), device="none")
+    ok = np.zeros((8, 9, 10))
+    with _pt.raises(ValueError, match="elements"):
+        plan.apply_host([np.zeros((8, 9, 9)), ok], scalars=[4.0, 0.5, 0.25])
+    r4 = sdag.Plan(sdag.spec_text("rhs4center"), (8, 9, 10), device="none")
+    g = [np.zeros((8, 9, 10)) for _ in range(8)]
+    with _pt.raises(ValueError, match="axis"):
+        r4.apply_host(g, [np.zeros(10), np.zeros(9), np.zeros(9)], scalars=[0.75, 1 / 6, 1 / 144, 1.0, 1.0])

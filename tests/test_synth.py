@@ -22,3 +22,22 @@ def test_uniform_torch_matches_numpy():
     if torch.cuda.is_available():  # pragma: no cover
         c = synth.uniform_torch((9, 10, 11), 0.5, 1.5, "t", "A", device="cuda")
         assert np.array_equal(a, c.cpu().numpy())
+
+
+def test_recipes_match_the_input_builders():
+    """bench.py builds BASELINE inputs on the device from synth.recipe(); they
+    are bit-identical to the *_inputs() arrays the parity tests use."""
+    dims = (5, 6, 7)
+    builders = {"jacobi7": synth.jacobi7_inputs, "lap25": synth.lap25_inputs, "smooth27": synth.smooth27_inputs,
+                "hypterm": synth.hypterm_inputs, "rhs4center": synth.rhs4_inputs}
+    for name, fn in builders.items():
+        cfg, a3, a1, sc = synth.recipe(name)
+        ins, sc_ref = fn(dims, cfg=cfg)
+        assert sc == sc_ref, name
+        assert set(ins) == set(a3) | set(a1), name
+        for k, (lo, hi) in a3.items():
+            t = synth.uniform_torch(dims, lo, hi, cfg, k, device="cpu")
+            assert np.array_equal(t.numpy(), ins[k]), (name, k)
+        for k, (lo, hi) in a1.items():
+            n = {"strx": dims[2], "stry": dims[1], "strz": dims[0]}[k]
+            assert np.array_equal(synth.uniform((n,), lo, hi, cfg, k), ins[k]), (name, k)
