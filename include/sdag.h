@@ -391,6 +391,43 @@ sdag_status sdag_spec_fission(const char *spec, int32_t kind, char *buf, int64_t
  * arrays read by a later stage are not written (only the sinks).  UNSUPPORTED
  * when a written array is also read at an offset before any stage writes it.
  * Buffer convention as sdag_spec_fission.  Host only. */
+/* Section VI-B versions of a multi-stencil program, as DSL text
+ * with the program's arguments unchanged (declaration order):
+ *   SDAG_VERSION_MAXFUSE    all calls fused into one stencil with recomputation
+ *                           (intermediates only read inside are not written);
+ *   SDAG_VERSION_STAGED     every call its own stencil (the program re-printed);
+ *   SDAG_VERSION_RECOMPUTE  recompute-fission: calls grouped in call order, each
+ *                           group grown while its recomputation halo stays
+ *                           <= max(4, r), r the largest order of its calls
+ *                           (P:1538-1544); the group sizes are written to
+ *                           sizes[] (capacity n_sizes) if non-null;
+ *   SDAG_VERSION_GROUPS     the calls grouped as sizes[0..n_sizes) (sum = number
+ *                           of calls), each group fused.
+ * A fused group writes the arrays later groups read and the program's results
+ * on ITS composed interior, where every value is computed by the operations of
+ * the staged program (reading R24).  Buffer convention as sdag_spec_fission.
+ * UNSUPPORTED when a group would read an array it writes at an offset.  Host only. */
+enum { SDAG_VERSION_MAXFUSE = 0, SDAG_VERSION_STAGED = 1, SDAG_VERSION_RECOMPUTE = 2, SDAG_VERSION_GROUPS = 3 };
+sdag_status sdag_program_version(const char *program, int32_t kind, int32_t *sizes, int32_t n_sizes, char *buf,
+                                 int64_t cap, int64_t *len);
+/* The fusion forest: every partition of the calls into contiguous
+ * groups whose recomputation halo is <= max(4, r) and which recompute at most 4
+ * RAW intermediates -- the staged program first, maxfuse last when allowed.
+ * Candidate c has n_groups[c] groups of sizes sizes[c * 16 + g].  At most
+ * max_candidates are returned (*n_candidates); programs of > 16 calls are
+ * UNSUPPORTED.  Host only. */
+sdag_status sdag_program_forest(const char *program, int32_t max_candidates, int32_t *n_groups, int32_t *sizes,
+                                int32_t *n_candidates);
+/* The measured pick among the forest's candidates (ARTEMIS's tuning of the
+ * fission versions): each candidate is planned (opts as
+ * sdag_program_create) and timed on the caller's arrays (device pointers,
+ * program argument order; outputs are overwritten) with CUDA events, median of
+ * 5 runs after 2 warm-ups; ms[c] receives candidate c's time (capacity
+ * max_candidates) and *best the fastest.  Synchronous. */
+sdag_status sdag_program_forest_tune(const char *program, const int64_t dims[3], const sdag_plan_opts *opts,
+                                     void *const *arrays3d, int32_t n3d, const double *const *arrays1d,
+                                     int32_t n1d, const double *scalars, int32_t nscalars, sdag_stream stream,
+                                     int32_t max_candidates, double *ms, int32_t *n_candidates, int32_t *best);
 sdag_status sdag_program_fuse(const char *program, int32_t keep_intermediates, char *buf, int64_t cap,
                               int64_t *len);
 

@@ -21,7 +21,8 @@ import os
 from . import _capi
 from ._capi import PlanInfo, PlanOpts, SDAG_DEVICE_CURRENT, SDAG_DEVICE_NONE
 
-__all__ = ["Plan", "Program", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "slab_partition2", "slab_halo2", "fission", "fuse_program", "nccl_unique_id",
+__all__ = ["Plan", "Program", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "slab_partition2", "slab_halo2", "fission", "fuse_program", "program_version", "program_forest",
+           "program_forest_tune", "nccl_unique_id",
            "nccl_comm_create", "nccl_comm_destroy", "launch_count", "fp64_peak", "version", "SPEC_DIR"]
 
 SPEC_DIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "specs")
@@ -563,6 +564,58 @@ def fuse_program(program: str, keep_intermediates: bool = True) -> str:
     buf = ctypes.create_string_buffer(n.value + 1)
     _check(L.sdag_program_fuse(program.encode(), int(keep_intermediates), buf, n.value + 1, ctypes.byref(n)))
     return buf.value.decode()
+
+
+_VERSION = {"maxfuse": 0, "staged": 1, "recompute": 2, "groups": 3}
+
+
+def program_version(program: str, kind: str = "recompute", groups=None):
+    """Section VI-B versions of a multi-stencil program (sdag_program_version):
+    kind "maxfuse", "staged", "recompute" (recompute-fission: groups grown while
+    the recomputation halo <= max(4, r)) or "groups" (fuse the calls in groups
+    of the given sizes).  Returns (DSL text, group sizes)."""
+    L = _capi.lib()
+    k = _VERSION[kind]
+    if kind == "groups":
+        sizes = (ctypes.c_int32 * len(groups))(*[int(x) for x in groups])
+        ns = len(groups)
+    else:
+        sizes = (ctypes.c_int32 * 16)()
+        ns = 16
+    n = ctypes.c_int64()
+    _check(L.sdag_program_version(program.encode(), k, sizes, ns, None, 0, ctypes.byref(n)))
+    buf = ctypes.create_string_buffer(n.value + 1)
+    _check(L.sdag_program_version(program.encode(), k, sizes, ns, buf, n.value + 1, ctypes.byref(n)))
+    g = list(groups) if kind == "groups" else [x for x in sizes if x] if kind == "recompute" else None
+    return buf.value.decode(), g
+
+
+def program_forest(program: str, max_candidates: int = 64):
+    """The fusion forest's candidates (sdag_program_forest): list of group-size lists"""
+    L = _capi.lib()
+    ng = (ctypes.c_int32 * max_candidates)()
+    sz = (ctypes.c_int32 * (16 * max_candidates))()
+    n = ctypes.c_int32()
+    _check(L.sdag_program_forest(program.encode(), int(max_candidates), ng, sz, ctypes.byref(n)))
+    return [[sz[c * 16 + g] for g in range(ng[c])] for c in range(n.value)]
+
+
+def program_forest_tune(program: str, dims, arrays3d, arrays1d=(), scalars=(), stream=None, max_candidates=64,
+                        device=None, tune=False):
+    """Time every forest candidate on these arrays (program argument order;
+    outputs overwritten): (candidates, ms per candidate, index of the fastest)"""
+    L = _capi.lib()
+    d = (ctypes.c_int64 * 3)(*[int(x) for x in dims])
+    o = _opts(-1, device, tune, 1, None, True)
+    p3 = [_ptr(t, "grid array") for t in arrays3d]
+    p1 = [_ptr(t, "1D array") for t in arrays1d]
+    s, ns = _scal(scalars)
+    ms = (ctypes.c_double * max_candidates)()
+    n, best = ctypes.c_int32(), ctypes.c_int32()
+    _check(L.sdag_program_forest_tune(program.encode(), d, ctypes.byref(o), _arr(p3), len(p3), _arr(p1), len(p1), s,
+                                      ns, _stream_handle(stream), int(max_candidates), ms, ctypes.byref(n),
+                                      ctypes.byref(best)))
+    return program_forest(program, max_candidates), list(ms[:n.value]), best.value
 
 
 def launch_count() -> int:

@@ -95,6 +95,13 @@ def lib():
                                          c_i32, P, c_i64p, c_i64p]),
             "sdag_spec_fission": (S, [c_char_p, c_i32, ctypes.c_char_p, c_i64, c_i64p]),
             "sdag_program_fuse": (S, [c_char_p, c_i32, ctypes.c_char_p, c_i64, c_i64p]),
+            "sdag_program_version": (S, [c_char_p, c_i32, ctypes.POINTER(c_i32), c_i32, ctypes.c_char_p, c_i64,
+                                         c_i64p]),
+            "sdag_program_forest": (S, [c_char_p, c_i32, ctypes.POINTER(c_i32), ctypes.POINTER(c_i32),
+                                        ctypes.POINTER(c_i32)]),
+            "sdag_program_forest_tune": (S, [c_char_p, c_i64p, ctypes.POINTER(PlanOpts), ctypes.POINTER(c_void_p),
+                                             c_i32, ctypes.POINTER(c_void_p), c_i32, c_dblp, c_i32, P, c_i32,
+                                             c_dblp, ctypes.POINTER(c_i32), ctypes.POINTER(c_i32)]),
             "sdag_plan_profile": (S, [P, ctypes.POINTER(c_void_p), c_i32, ctypes.POINTER(c_void_p), c_i32, c_dblp,
                                       c_i32, ctypes.c_double, ctypes.c_double, P, ctypes.c_void_p]),
             "sdag_dist_p2p_alloc": (S, [P, ctypes.POINTER(c_void_p), ctypes.POINTER(c_void_p)]),
@@ -138,7 +145,7 @@ EXPORTED = [
     "sdag_slab_partition2", "sdag_slab_halo2", "sdag_nccl_get_unique_id", "sdag_nccl_comm_create",
     "sdag_nccl_comm_destroy", "sdag_dist_create", "sdag_dist_layout", "sdag_dist_alloc_dims", "sdag_dist_local_plan", "sdag_dist_apply",
     "sdag_dist_apply_iterated", "sdag_dist_destroy", "sdag_dist_apply_host", "sdag_dist_apply_iterated_loopback",
-    "sdag_spec_fission", "sdag_program_fuse", "sdag_plan_profile", "sdag_dist_p2p_alloc", "sdag_dist_p2p_handle", "sdag_dist_p2p_attach", "sdag_dist_p2p_attach_local",
+    "sdag_spec_fission", "sdag_program_version", "sdag_program_forest", "sdag_program_forest_tune", "sdag_program_fuse", "sdag_plan_profile", "sdag_dist_p2p_alloc", "sdag_dist_p2p_handle", "sdag_dist_p2p_attach", "sdag_dist_p2p_attach_local",
     "sdag_dist_p2p_apply_iterated", "sdag_last_error",
     "sdag_version", "sdag_launch_count", "sdag_measure_fp64_peak", "sdag_registry_count", "sdag_registry_get",
 ]

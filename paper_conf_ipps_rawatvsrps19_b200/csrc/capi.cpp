@@ -402,6 +402,65 @@ sdag_status sdag_program_fuse(const char *program, int32_t keep, char *buf, int6
     });
 }
 
+sdag_status sdag_program_version(const char *program, int32_t kind, int32_t *sizes, int32_t n_sizes, char *buf,
+                                 int64_t cap, int64_t *len) {
+    return guard([&] {
+        if (!program || !len) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null argument");
+        std::string t;
+        const sdag::ProgramIR ir = sdag::parse_program(program);
+        const int nst = int(ir.stages.size());
+        if (kind == SDAG_VERSION_MAXFUSE) {
+            t = sdag::fuse_groups(program, std::vector<int>{nst});
+        } else if (kind == SDAG_VERSION_STAGED) {
+            t = sdag::fuse_groups(program, std::vector<int>(nst, 1));
+        } else if (kind == SDAG_VERSION_RECOMPUTE) {
+            std::vector<int> g;
+            t = sdag::recompute_fission(program, &g);
+            if (sizes)
+                for (int q = 0; q < n_sizes; q++) sizes[q] = q < int(g.size()) ? g[q] : 0;
+        } else if (kind == SDAG_VERSION_GROUPS) {
+            if (!sizes || n_sizes < 1) throw sdag::Error(SDAG_ERR_INVALID_ARG, "group sizes needed");
+            t = sdag::fuse_groups(program, std::vector<int>(sizes, sizes + n_sizes));
+        } else {
+            throw sdag::Error(SDAG_ERR_INVALID_ARG, "unknown version kind");
+        }
+        *len = int64_t(t.size());
+        if (buf) {
+            if (cap <= *len) throw sdag::Error(SDAG_ERR_INVALID_ARG, "buffer too small");
+            std::memcpy(buf, t.c_str(), t.size() + 1);
+        }
+    });
+}
+
+sdag_status sdag_program_forest(const char *program, int32_t max_candidates, int32_t *n_groups, int32_t *sizes,
+                                int32_t *n_candidates) {
+    return guard([&] {
+        if (!program || !n_candidates || max_candidates < 1) throw sdag::Error(SDAG_ERR_INVALID_ARG, "bad argument");
+        const auto c = sdag::forest_partitions(program, max_candidates);
+        *n_candidates = int32_t(c.size());
+        for (size_t q = 0; q < c.size(); q++) {
+            if (n_groups) n_groups[q] = int32_t(c[q].size());
+            if (sizes)
+                for (int g = 0; g < 16; g++) sizes[q * 16 + g] = g < int(c[q].size()) ? c[q][g] : 0;
+        }
+    });
+}
+
+sdag_status sdag_program_forest_tune(const char *program, const int64_t dims[3], const sdag_plan_opts *opts,
+                                     void *const *a3, int32_t n3, const double *const *a1, int32_t n1,
+                                     const double *s, int32_t ns, sdag_stream stream, int32_t max_candidates,
+                                     double *ms, int32_t *n_candidates, int32_t *best) {
+    return guard([&] {
+        if (!program || !dims || !n_candidates || !best || max_candidates < 1)
+            throw sdag::Error(SDAG_ERR_INVALID_ARG, "bad argument");
+        sdag_plan_opts o;
+        sdag_plan_opts_init(&o);
+        if (opts) o = *opts;
+        sdag::program_forest_tune(program, dims, o, reinterpret_cast<double *const *>(a3), n3, a1, n1, s, ns,
+                                  reinterpret_cast<cudaStream_t>(stream), max_candidates, ms, n_candidates, best);
+    });
+}
+
 sdag_status sdag_plan_profile(sdag_plan plan, void *const *a3, int32_t n3, const double *const *a1, int32_t n1,
                               const double *s, int32_t ns, double peak_hbm_gbs, double peak_fp64_tflops,
                               sdag_stream stream, sdag_profile *out) {

@@ -18,6 +18,7 @@
 // parsed tree, fully parenthesised, literals printed to round-trip exactly.
 #include <algorithm>
 #include <cstdio>
+#include <functional>
 #include <set>
 #include <sstream>
 
@@ -269,7 +270,7 @@ namespace {
 struct Fuser {
     const ProgramIR &ir;
     std::vector<std::string> iters;
-    std::vector<int> writer_end;  // per program arg: not used
+    int s0 = 0;  // first stage of the fused group: earlier stages' results are read from memory
 
     const std::string &argname(int s, int formal_pos) const { return ir.args[ir.map[s][formal_pos]].name; }
     int arg_of(int s, ArgKind k, int kind_index) const {
@@ -300,7 +301,7 @@ struct Fuser {
     std::string value(int s, int q, int a, const int d[3], const std::vector<bool> &fused_writes) const {
         const int w = last_write(s, a, q);
         if (w >= 0) return "(" + expr(s, w, ir.stages[s].stmts[w].expr, d, fused_writes) + ")";
-        for (int e = s - 1; e >= 0; e--) {  // the last earlier stage that wrote a
+        for (int e = s - 1; e >= s0; e--) {  // the last earlier stage of the group that wrote a
             const int we = last_write(e, a, int(ir.stages[e].stmts.size()));
             if (we >= 0) return "(" + expr(e, we, ir.stages[e].stmts[we].expr, d, fused_writes) + ")";
         }
@@ -353,7 +354,7 @@ std::string fuse_program(const std::string &text, int keep_intermediates) {
         if (st.iterators != ir.stages[0].iterators || st.iterators.size() != 3)
             throw Error(SDAG_ERR_UNSUPPORTED, "fuse: stages must share three iterators");
     }
-    Fuser F{ir, ir.stages[0].iterators, {}};
+    Fuser F{ir, ir.stages[0].iterators, 0};
     const int na = int(ir.args.size());
     // arrays some stage writes, in order of their last write; read later?
     std::vector<bool> written(na, false), read_later(na, false);
@@ -404,6 +405,261 @@ std::string fuse_program(const std::string &text, int keep_intermediates) {
     o << "}\nfused (";
     for (int a = 0; a < na; a++) o << (a ? ", " : "") << ir.args[a].name;
     o << ");\n";
+    return o.str();
+}
+
+
+// ---------------------------------------------------------------------------
+// Recompute-fission and the fusion forest (Section VI-B).
+//
+// A version of a multi-stencil program is a partition of its calls (in call
+// order) into contiguous groups -- the trees of the paper's forest; each group
+// becomes one stencil, fused with recomputation as fuse_program does (a read
+// of an array written earlier IN THE GROUP is replaced by the writer's
+// expression at the read's offset; arrays written by earlier groups are read
+// from memory).  A group writes the arrays a later group reads, and every
+// array no later stage reads (the program's results); intermediates consumed
+// only inside the group never go through memory.
+//
+// Per group (group_info): r = the largest stencil order (radius, reading R2)
+// of its calls; halo = the recomputation halo: how far beyond an output point
+// an intermediate of the group must be recomputed (a chain lap(lap(A)) of
+// order-1 calls: 1); raw = the number of intermediates the group reads at a
+// nonzero offset (the "RAW dependences that increase recomputation volume").
+// recompute-fission: grow each group in call order while its
+// halo stays <= max(4, r).  The forest search enumerates every
+// partition whose groups have halo <= max(4, r) and raw <= 4 -- maxfuse, the
+// staged program and everything between -- for the measured pick.
+// ---------------------------------------------------------------------------
+
+namespace {
+
+struct Grp {
+    int halo = 0, r = 0, raw = 0;
+    bool ok = true;
+};
+
+Grp group_info(const ProgramIR &ir, int s0, int s1) {
+    Fuser F{ir, ir.stages[0].iterators, s0};
+    const int na = int(ir.args.size());
+    Grp g;
+    std::vector<int> need(na, -1);  // halo at which a group-internal array's values are needed
+    std::vector<bool> written(na, false);
+    for (int s = s0; s < s1; s++) {
+        const Stencil &st = ir.stages[s];
+        const Analysis an = analyse(st);
+        g.r = std::max({g.r, an.radius[0], an.radius[1], an.radius[2]});
+    }
+    // arrays read by a later stage of the group (intermediates) and their writers
+    std::vector<int> writer(na, -1);
+    for (int s = s0; s < s1; s++)
+        for (const Statement &w : ir.stages[s].stmts)
+            if (w.to_array) writer[F.arg_of(s, ArgKind::Array3D, w.target)] = s;
+    // reverse pass: a stage runs wherever one of its outputs is needed
+    std::vector<int> stage_need(s1, 0);
+    for (int s = s1 - 1; s >= s0; s--) {
+        const Stencil &st = ir.stages[s];
+        int ns = 0;
+        for (const Statement &w : st.stmts)
+            if (w.to_array) {
+                const int a = F.arg_of(s, ArgKind::Array3D, w.target);
+                if (need[a] > ns) ns = need[a];
+            }
+        stage_need[s] = ns;
+        std::set<int> raw_here;
+        for (const Node &n : st.nodes) {
+            if (n.kind != Node::Load3) continue;
+            const int a = F.arg_of(s, ArgKind::Array3D, n.ref);
+            int e = -1;  // the group's last writer of a before stage s
+            for (int q = s - 1; q >= s0; q--)
+                if (F.last_write(q, a, int(ir.stages[q].stmts.size())) >= 0) {
+                    e = q;
+                    break;
+                }
+            if (e < 0) continue;
+            const int d = std::max({std::abs(n.off[0]), std::abs(n.off[1]), std::abs(n.off[2])});
+            need[a] = std::max(need[a], ns + d);
+            if (d > 0) raw_here.insert(a);
+        }
+        g.raw += int(raw_here.size());
+    }
+    for (int a = 0; a < na; a++)
+        if (need[a] > g.halo) g.halo = need[a];
+    return g;
+}
+
+bool group_fusable(const ProgramIR &ir, int s0, int s1, Grp *out) {
+    Grp g = group_info(ir, s0, s1);
+    if (out) *out = g;
+    if (s1 - s0 == 1) return true;
+    return g.halo <= std::max(4, g.r) && g.raw <= 4;
+}
+
+// the group's stencil text (function `name`, formals = every program argument)
+std::string group_function(const ProgramIR &ir, int s0, int s1, const std::string &name) {
+    Fuser F{ir, ir.stages[0].iterators, s0};
+    const int na = int(ir.args.size());
+    std::vector<bool> written(na, false), read_after(na, false);
+    for (int s = s0; s < s1; s++)
+        for (const Statement &w : ir.stages[s].stmts)
+            if (w.to_array) written[F.arg_of(s, ArgKind::Array3D, w.target)] = true;
+    for (size_t s = s1; s < ir.stages.size(); s++)
+        for (const Node &n : ir.stages[s].nodes)
+            if (n.kind == Node::Load3) read_after[F.arg_of(int(s), ArgKind::Array3D, n.ref)] = true;
+    // inside the group, is a read by a later stage of the group -> intermediate
+    std::vector<bool> read_in_group(na, false);
+    for (int s = s0; s < s1; s++)
+        for (const Node &n : ir.stages[s].nodes)
+            if (n.kind == Node::Load3) {
+                const int a = F.arg_of(s, ArgKind::Array3D, n.ref);
+                for (int q = s0; q < s; q++)
+                    if (F.last_write(q, a, int(ir.stages[q].stmts.size())) >= 0) read_in_group[a] = true;
+            }
+    std::vector<bool> fw(na, false);
+    for (int a = 0; a < na; a++) fw[a] = written[a] && (read_after[a] || !read_in_group[a]);
+    std::ostringstream o;
+    o << "stencil " << name << " (";
+    for (int a = 0; a < na; a++) o << (a ? ", " : "") << ir.args[a].name;
+    o << ") {\n";
+    const int zero[3] = {0, 0, 0};
+    for (int a = 0; a < na; a++) {
+        if (!fw[a]) continue;
+        for (int s = s1 - 1; s >= s0; s--) {
+            const int w = F.last_write(s, a, int(ir.stages[s].stmts.size()));
+            if (w < 0) continue;
+            o << "    " << ir.args[a].name << "[" << F.iters[0] << "][" << F.iters[1] << "][" << F.iters[2]
+              << "] = " << F.expr(s, w, ir.stages[s].stmts[w].expr, zero, fw) << ";\n";
+            break;
+        }
+    }
+    o << "}\n";
+    return o.str();
+}
+
+std::string program_of_groups(const ProgramIR &ir, const std::vector<int> &sizes) {
+    const auto &it = ir.stages[0].iterators;
+    std::ostringstream o;
+    o << "iterator " << it[0] << ", " << it[1] << ", " << it[2] << ";\ndouble";
+    bool first = true;
+    for (const ProgramArg &a : ir.args) {
+        o << (first ? " " : ", ") << a.name;
+        if (a.kind == ArgKind::Array3D) o << "[64,64,64]";
+        if (a.kind == ArgKind::Array1D) o << "[64]";
+        first = false;
+    }
+    o << ";\n";
+    int s0 = 0, gi = 0;
+    std::ostringstream calls;
+    for (int n : sizes) {
+        const std::string name = "g" + std::to_string(gi++);
+        if (n == 1) {  // an unfused call: the stage itself, statements and temporaries as written
+            const Stencil &st = ir.stages[s0];
+            o << function(st, name, std::vector<bool>(st.stmts.size(), true));
+            calls << name << " " << formals_list(st, true) << ";\n";
+        } else {
+            o << group_function(ir, s0, s0 + n, name);
+            calls << name << " (";
+            for (size_t a = 0; a < ir.args.size(); a++) calls << (a ? ", " : "") << ir.args[a].name;
+            calls << ");\n";
+        }
+        s0 += n;
+    }
+    o << calls.str();
+    return o.str();
+}
+
+ProgramIR checked_program(const std::string &text) {
+    ProgramIR ir = parse_program(text);
+    if (ir.stages.empty()) throw Error(SDAG_ERR_INVALID_ARG, "empty program");
+    for (const Stencil &st : ir.stages) {
+        (void)analyse(st);
+        if (st.iterators != ir.stages[0].iterators || st.iterators.size() != 3)
+            throw Error(SDAG_ERR_UNSUPPORTED, "stages must share three iterators");
+    }
+    return ir;
+}
+
+}  // namespace
+
+std::string fuse_groups(const std::string &text, const std::vector<int> &sizes) {
+    const ProgramIR ir = checked_program(text);
+    int n = 0;
+    for (int x : sizes) {
+        if (x < 1) throw Error(SDAG_ERR_INVALID_ARG, "group sizes must be >= 1");
+        n += x;
+    }
+    if (n != int(ir.stages.size()))
+        throw Error(SDAG_ERR_INVALID_ARG, "group sizes must add up to the number of calls (" +
+                                              std::to_string(ir.stages.size()) + ")");
+    const std::string out = program_of_groups(ir, sizes);
+    (void)checked_program(out);  // every group must be a valid stencil (e.g. no shifted self-reads)
+    return out;
+}
+
+std::string recompute_fission(const std::string &text, std::vector<int> *sizes_out) {
+    const ProgramIR ir = checked_program(text);
+    const int ns = int(ir.stages.size());
+    std::vector<int> sizes;
+    int s0 = 0;
+    while (s0 < ns) {
+        int s1 = s0 + 1;
+        while (s1 < ns && group_fusable(ir, s0, s1 + 1, nullptr)) {
+            // the grown group must still be a valid fused stencil
+            try {
+                std::vector<int> trial(sizes);
+                trial.push_back(s1 + 1 - s0);
+                int rest = ns - (s1 + 1);
+                for (int q = 0; q < rest; q++) trial.push_back(1);
+                (void)checked_program(program_of_groups(ir, trial));
+            } catch (const Error &) {
+                break;
+            }
+            s1++;
+        }
+        sizes.push_back(s1 - s0);
+        s0 = s1;
+    }
+    if (sizes_out) *sizes_out = sizes;
+    return program_of_groups(ir, sizes);
+}
+
+std::vector<std::vector<int>> forest_partitions(const std::string &text, int max_candidates) {
+    const ProgramIR ir = checked_program(text);
+    const int ns = int(ir.stages.size());
+    if (ns > 16) throw Error(SDAG_ERR_UNSUPPORTED, "forest search: more than 16 calls");
+    std::vector<std::vector<int>> out;
+    // every composition of ns into contiguous groups, staged first, maxfuse last
+    std::vector<int> cur;
+    std::function<void(int)> rec = [&](int s0) {
+        if (int(out.size()) >= max_candidates) return;
+        if (s0 == ns) {
+            try {
+                (void)checked_program(program_of_groups(ir, cur));
+                out.push_back(cur);
+            } catch (const Error &) {
+            }
+            return;
+        }
+        for (int n = 1; s0 + n <= ns; n++) {
+            if (!group_fusable(ir, s0, s0 + n, nullptr)) break;
+            cur.push_back(n);
+            rec(s0 + n);
+            cur.pop_back();
+        }
+    };
+    rec(0);
+    return out;
+}
+
+std::string group_report(const std::string &text, const std::vector<int> &sizes) {
+    const ProgramIR ir = checked_program(text);
+    std::ostringstream o;
+    int s0 = 0;
+    for (int n : sizes) {
+        Grp g = group_info(ir, s0, s0 + n);
+        o << "[" << s0 << "," << s0 + n << ") r=" << g.r << " halo=" << g.halo << " raw=" << g.raw << "\n";
+        s0 += n;
+    }
     return o.str();
 }
 

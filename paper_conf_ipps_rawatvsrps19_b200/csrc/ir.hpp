@@ -130,6 +130,15 @@ std::string emit_fission(const std::string &spec, int kind);
 // maxfuse of a multi-stencil program with recomputation (fission.cpp): one
 // stencil; keep_intermediates = 0 writes only arrays no later stage reads
 std::string fuse_program(const std::string &text, int keep_intermediates);
+// Section VI-B versions of a multi-stencil program (fission.cpp): calls grouped
+// in call order (sizes add up to the number of calls), each group fused with
+// recomputation; recompute-fission = groups grown while the recomputation halo
+// <= max(4, r); forest_partitions = every partition whose groups obey that bound
+// and have <= 4 recomputed RAW intermediates (staged first, maxfuse last)
+std::string fuse_groups(const std::string &text, const std::vector<int> &sizes);
+std::string recompute_fission(const std::string &text, std::vector<int> *sizes_out);
+std::vector<std::vector<int>> forest_partitions(const std::string &text, int max_candidates);
+std::string group_report(const std::string &text, const std::vector<int> &sizes);
 // canonical, name-free serialisation used to match registered DAGs
 std::string canonical_form(const Stencil &st);
 

@@ -7,6 +7,10 @@ void add_kernels_rhs4(std::vector<KernelDesc> &v) {
     // specialised kernel (rhs4.cuh): 2 x UY patches from 128-bit pair loads, derivative fields
     // (2 x 2 / 2 x 4 patches spill at 255 registers and run 3x slower; not registered)
     SDAG_RHS4_PAIR(v, "rhs4center", 32, 16, 1, 1, -10);
+    // cooperative derivative fields + retimed z (rhs4f.cuh)
+    SDAG_RHS4F_PAIR(v, "rhs4center", 32, 16, 1, -3);
+    SDAG_RHS4F_PAIR(v, "rhs4center", 32, 8, 1, -2);
+    SDAG_RHS4G_PAIR(v, "rhs4center", 32, 16, -1);  // double-buffered fields, one barrier per plane
     SDAG_RHS4_PAIR(v, "rhs4center", 16, 16, 1, 1, -9);
     SDAG_RHS4_PAIR(v, "rhs4center", 64, 8, 1, 1, -8);
     SDAG_RHS4_PAIR(v, "rhs4center", 32, 8, 1, 1, -7);

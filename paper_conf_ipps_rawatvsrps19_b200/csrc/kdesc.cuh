@@ -11,6 +11,7 @@
 #include "fuseN.cuh"
 #include "hyp.cuh"
 #include "rhs4.cuh"
+#include "rhs4f.cuh"
 #include "star.cuh"
 #include "sweep.cuh"
 
@@ -219,6 +220,31 @@ KernelDesc make_rhs4_desc(const char *dag, int prio) {
     d.prio = prio;
     return d;
 }
+
+// rhs4center with cooperative derivative fields (rhs4f.cuh)
+template <int TX, int TY, int PF, bool TMA, int FB = 1>
+KernelDesc make_rhs4f_desc(const char *dag, int prio) {
+    using G = dev::R4fGeo<TX, TY, PF, FB>;
+    KernelDesc d = make_rhs4_desc<TX, TY, 1, PF, TMA>(dag, prio);
+    char buf[96];
+    std::snprintf(buf, sizeof buf, "r4%s_%s_%dx%d_u2x1_pf%d", FB == 2 ? "g" : "f", TMA ? "tma" : "lsu", TX, TY, PF);
+    d.variant = buf;
+    d.fn = reinterpret_cast<const void *>(&dev::sdag_rhs4f<TX, TY, PF, TMA, FB>);
+    d.threads = G::THREADS;
+    d.smem = G::SMEM;
+    return d;
+}
+
+#define SDAG_RHS4F_PAIR(v, DAG, TX, TY, PF, PRIO)                                  \
+    do {                                                                           \
+        v.push_back(make_rhs4f_desc<TX, TY, PF, true>(DAG, PRIO));                 \
+        v.push_back(make_rhs4f_desc<TX, TY, PF, false>(DAG, PRIO + 100));          \
+    } while (0)
+#define SDAG_RHS4G_PAIR(v, DAG, TX, TY, PRIO)                                      \
+    do {                                                                           \
+        v.push_back(make_rhs4f_desc<TX, TY, 0, true, 2>(DAG, PRIO));               \
+        v.push_back(make_rhs4f_desc<TX, TY, 0, false, 2>(DAG, PRIO + 100));        \
+    } while (0)
 
 #define SDAG_RHS4_PAIR(v, DAG, TX, TY, UY, PF, PRIO)                               \
     do {                                                                           \

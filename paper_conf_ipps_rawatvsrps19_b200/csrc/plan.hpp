@@ -108,6 +108,10 @@ Program *program_create(const std::string &spec, const int64_t dims[3], const sd
 void program_apply(Program *g, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns,
                    int batch, cudaStream_t stream);
 void plan_fill_info(Plan *p, sdag_plan_info *info);
+// the fusion forest's measured pick (program.cpp, Section VI-B)
+void program_forest_tune(const std::string &text, const int64_t dims[3], const sdag_plan_opts &o, double *const *a3,
+                         int n3, const double *const *a1, int n1, const double *s, int ns, cudaStream_t stream,
+                         int max_candidates, double *ms, int *n_candidates, int *best);
 
 // Peer-memory halo of one launch (dist p2p path): output planes [klo[s], khi[s])
 // are also stored into neighbour s's buffer `peer[s]` at element offset

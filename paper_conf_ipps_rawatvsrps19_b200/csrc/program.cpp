@@ -12,6 +12,7 @@
 // declarations); a stage's formal q is program argument map[s][q].
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <memory>
 #include <string>
 #include <vector>
@@ -88,6 +89,43 @@ void program_apply(Program *g, double *const *a3, int n3, const double *const *a
     for (size_t st = 0; st < g->stages.size(); st++)
         apply(g->stages[st].get(), b[st].a3.data(), int(b[st].a3.size()), b[st].a1.data(), int(b[st].a1.size()),
               b[st].s.data(), int(b[st].s.size()), batch, stream);
+}
+
+// Section VI-B: time every fusion-forest candidate of the program on the
+// caller's arrays and report the fastest (the paper's tuning over fission
+// versions).  Every candidate keeps the program's arguments.
+void program_forest_tune(const std::string &text, const int64_t dims[3], const sdag_plan_opts &o, double *const *a3,
+                         int n3, const double *const *a1, int n1, const double *s, int ns, cudaStream_t stream,
+                         int max_candidates, double *ms, int *n_candidates, int *best) {
+    const auto cands = forest_partitions(text, max_candidates);
+    *n_candidates = int(cands.size());
+    *best = -1;
+    double best_ms = 0.0;
+    cudaEvent_t e0, e1;
+    check_cuda(cudaEventCreate(&e0), "cudaEventCreate");
+    check_cuda(cudaEventCreate(&e1), "cudaEventCreate");
+    for (size_t c = 0; c < cands.size(); c++) {
+        std::unique_ptr<Program> g(program_create(fuse_groups(text, cands[c]), dims, o));
+        std::vector<float> t;
+        for (int it = 0; it < 7; it++) {
+            check_cuda(cudaEventRecord(e0, stream), "cudaEventRecord");
+            program_apply(g.get(), a3, n3, a1, n1, s, ns, 1, stream);
+            check_cuda(cudaEventRecord(e1, stream), "cudaEventRecord");
+            check_cuda(cudaEventSynchronize(e1), "cudaEventSynchronize");
+            float x = 0.f;
+            check_cuda(cudaEventElapsedTime(&x, e0, e1), "cudaEventElapsedTime");
+            if (it >= 2) t.push_back(x);
+        }
+        std::sort(t.begin(), t.end());
+        const double med = t[t.size() / 2];
+        if (ms) ms[c] = med;
+        if (*best < 0 || med < best_ms) {
+            *best = int(c);
+            best_ms = med;
+        }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
 }
 
 }  // namespace sdag

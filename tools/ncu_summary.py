@@ -75,6 +75,10 @@ if __name__ == "__main__":
         x, u = num(k, n)
         if x is not None:
             res["metrics"][n] = {"value": x, "unit": u}
+    fp = [num(k, f"smsp__sass_thread_inst_executed_op_{o}_pred_on.sum")[0] for o in ("dfma", "dadd", "dmul")]
+    if all(x is not None for x in fp):
+        res["fp64_thread_inst_per_launch"] = {"dfma": fp[0], "dadd": fp[1], "dmul": fp[2]}
+        res["fp64_flops_executed_per_launch"] = 2 * fp[0] + fp[1] + fp[2]
     rb = num(k, "dram__bytes_read.sum")
     wb = num(k, "dram__bytes_write.sum")
     if rb[0] is not None and wb[0] is not None:
@@ -97,15 +101,19 @@ if __name__ == "__main__":
         for n, v in res["metrics"].items():
             f.write(f"| {n} | {v['value']:.6g} | {v['unit']} |\n")
         for n in ("dram_bytes_per_launch", "alg_bytes_per_launch", "traffic_over_alg", "alg_GBps_under_ncu",
-                  "GFLOPs_under_ncu"):
+                  "GFLOPs_under_ncu", "fp64_flops_executed_per_launch"):
             if n in res:
                 f.write(f"| {n} | {res[n]:.6g} | |\n")
         f.write("\nTop warp stall reasons (pc samples):\n\n")
         for n, v in res["stalls"].items():
             f.write(f"- {n}: {v}\n")
     if a.variant and "dram_bytes_per_launch" in res:
-        p = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "ncu_traffic.json")
+        # per-launch counters read by bench.py (roofline.traffic, the F = min(canonical, executed) rule)
+        p = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "ncu_counters.json")
         d = json.load(open(p)) if os.path.exists(p) else {}
-        d[a.variant] = res["dram_bytes_per_launch"]
+        e = {"dram_bytes": res["dram_bytes_per_launch"], "source": os.path.basename(a.report)}
+        if "fp64_flops_executed_per_launch" in res:
+            e["fp64_flops"] = res["fp64_flops_executed_per_launch"]
+        d[a.variant] = e
         json.dump(d, open(p, "w"), indent=1, sort_keys=True)
     print(json.dumps({k2: res[k2] for k2 in res if k2 != "metrics"}, indent=1))
