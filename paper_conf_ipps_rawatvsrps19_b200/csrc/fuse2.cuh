@@ -190,31 +190,22 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
                 if (zring || ringxy[py][px]) v[px] = A1[py][px];  // ring: not updated by sweep 1
                 A1[py][px] = s0[py][px];
             }
-            if constexpr (ODD) {
-                // the patch starts at an odd column: store ALIGNED pairs, the last
-                // one completed with the next lane's first value (a shuffle), so
-                // no 8-byte stores at a 16-byte lane stride (2-way bank conflict,
-                // ncu r02: 50 % excess wavefronts on these stores).  The last lane
-                // of a row puts its second value in the unused column past the
-                // region.
-                const double nxt = __shfl_down_sync(0xffffffffu, v[0], 1);
-                double *row = s1 + (cy + py + 1) * PX + cx + ML;
 #pragma unroll
-                for (int px = 1; px + 1 < UX; px += 2)
-                    *reinterpret_cast<double2 *>(row + px) = make_double2(v[px], v[px + 1]);
-                // lane 31 cannot see its right neighbour when a row spans two
-                // warps: it stores its own value only, lane 0 of the next warp
-                // (and of every row) its first one
-                if ((t & 31) == 31)
-                    row[UX - 1] = v[UX - 1];
-                else
-                    *reinterpret_cast<double2 *>(row + UX - 1) = make_double2(v[UX - 1], nxt);
-                if ((t & 31) == 0 || lx == 0) row[0] = v[0];
-            } else {
-#pragma unroll
-                for (int px = 0; px < UX; px += 2)
-                    *reinterpret_cast<double2 *>(s1 + (cy + py + 1) * PX + cx + ML + px) =
-                        make_double2(v[px], v[px + 1]);
+            for (int px = 0; px < UX; px += 2) {
+                double *q = s1 + (cy + py + 1) * PX + cx + ML + px;
+                if constexpr (ODD) {
+                    // two 8-byte stores at a 16-byte lane stride are 2-way bank
+                    // conflicted (ncu r02: 50 % excess wavefronts on these four
+                    // STS.64, 15 % of the kernel's).  Measured and reverted (r02):
+                    // aligned STS.128 pairs completed by a shuffle of the next
+                    // lane's value cut the conflicts 137 M -> 46 M per launch but
+                    // ran 4.51 -> 5.00 ms per launch: the store side is not the
+                    // bound, the fold's dependency chains are (issue 58 %).
+                    q[0] = v[px];
+                    q[1] = v[px + 1];
+                } else {
+                    *reinterpret_cast<double2 *>(q) = make_double2(v[px], v[px + 1]);
+                }
             }
         }
         __syncthreads();  // sweep-1 plane j is complete in shared memory
