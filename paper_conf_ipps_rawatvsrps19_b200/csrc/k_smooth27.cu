@@ -31,6 +31,10 @@ void add_kernels_smooth27(std::vector<KernelDesc> &v) {
     v.push_back(make_fuse2_desc<128, 16, 2, 2>("smooth27", 27));
     v.push_back(make_fuse2_desc<64, 16, 2, 2, 2, 4, true>("smooth27", 28));
     v.push_back(make_fuse2_desc<64, 16, 2, 2, 1, 4>("smooth27", 29));  // 4-wide patch: bank-conflicted, kept for comparison
+    // round 2, measured and removed (tools/fusion_sweep.py, 1024^3, T = 12, ms per
+    // sweep vs 2.39 for fuse2o 62x14 u2x2 mb2): 2x4 patches 62x14 mb3 2.94 (168 regs,
+    // spills), 62x22 mb2 3.05, 62x30 2.63 (224 regs, 8 warps/SM); 2x2 with 3 CTAs/SM
+    // (80 regs, spills) 3.82
     // fusion degrees 3 and 4 (fuseN.cuh): the paper's Table II / Fig 4 sweep
     v.push_back(make_fuseN_desc<3, 64, 32, 2, 2, 1, 2, false, 0>("smooth27", 40));
     v.back().fhint = 3.12;  // f(3): 1.04 per sweep -- past the cusp (shared-memory bound folds)
