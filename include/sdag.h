@@ -272,6 +272,14 @@ sdag_status sdag_nccl_comm_create(const uint8_t id[128], int32_t nranks, int32_t
                                   void **comm);
 void sdag_nccl_comm_destroy(void *comm);
 
+/* SURVEY 8(b)'s form: this rank's slab from a LOCAL plan of its owned planes
+ * (dims = nz_own, ny, nx), every rank owning nz_own planes (weak scaling:
+ * global nz = nz_own * nranks).  The plan must come from sdag_plan_create (its
+ * spec text and options are reused; the dist plans its own local layout with
+ * ghost planes, sdag_dist_layout); the caller keeps ownership of `local`.
+ * time_tile as opts.time_tile.  UNSUPPORTED for program stages. */
+sdag_status sdag_dist_create_local(sdag_plan local, int32_t rank, int32_t nranks, void *nccl_comm, int32_t time_tile,
+                                   sdag_dist *out);
 /* Create this rank's slab of a `global_dims` problem.  `nccl_comm` is an
  * ncclComm_t from sdag_nccl_comm_create (or NULL when nranks == 1). */
 sdag_status sdag_dist_create(const char *spec, const int64_t global_dims[3], const sdag_plan_opts *opts,

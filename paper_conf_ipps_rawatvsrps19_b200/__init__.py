@@ -425,6 +425,19 @@ class Dist:
         axes = [a[3] for a in self.plan.args() if a[0] == 1]
         _check_sizes(arrays3d, arrays1d, dims, axes, 1, self._device, host)
 
+    @classmethod
+    def from_local_plan(cls, plan: "Plan", rank, nranks, comm=None, time_tile=1):
+        """SURVEY 8(b)'s form: a dist from a plan of this rank's owned slab
+        (nz_own, ny, nx); global nz = nz_own * nranks (sdag_dist_create_local)"""
+        d = cls.__new__(cls)
+        d._L = _capi.lib()
+        d._h = ctypes.c_void_p()
+        _check(d._L.sdag_dist_create_local(plan._h, int(rank), int(nranks), ctypes.c_void_p(comm or 0),
+                                           int(time_tile), ctypes.byref(d._h)))
+        d.rank, d.nranks = rank, nranks
+        d._device = getattr(plan, "_device", None)
+        return d
+
     def close(self):
         if self._h:
             self._L.sdag_dist_destroy(self._h)

@@ -325,6 +325,14 @@ sdag_status sdag_dist_create(const char *spec, const int64_t global_dims[3], con
     });
 }
 
+sdag_status sdag_dist_create_local(sdag_plan local, int32_t rank, int32_t nranks, void *nccl_comm, int32_t time_tile,
+                                   sdag_dist *out) {
+    return guard([&] {
+        if (!local || !local->p || !out) throw sdag::Error(SDAG_ERR_INVALID_ARG, "null argument");
+        *out = reinterpret_cast<sdag_dist>(sdag::dist_create_local(local->p, rank, nranks, nccl_comm, time_tile));
+    });
+}
+
 sdag_status sdag_dist_layout(sdag_dist d, int64_t local_dims[3], int64_t *gz0) {
     return guard([&] {
         auto *D = reinterpret_cast<sdag::Dist *>(d);

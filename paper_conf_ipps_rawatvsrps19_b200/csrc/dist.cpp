@@ -199,6 +199,20 @@ Dist *dist_create(const std::string &spec, const int64_t gdims[3], const sdag_pl
     return d.release();
 }
 
+Dist *dist_create_local(const Plan *local, int rank, int nranks, void *comm, int time_tile) {
+    if (!local) throw Error(SDAG_ERR_INVALID_ARG, "null plan");
+    if (local->spec_text.empty())
+        throw Error(SDAG_ERR_UNSUPPORTED, "the plan was not created from spec text (a program stage)");
+    if (nranks < 1) throw Error(SDAG_ERR_INVALID_ARG, "nranks must be >= 1");
+    const int64_t g[3] = {local->dims[0] * nranks, local->dims[1], local->dims[2]};
+    sdag_plan_opts o = local->opts_copy;
+    o.force_variant = local->force_variant.empty() ? nullptr : local->force_variant.c_str();
+    o.time_tile = time_tile < 1 ? 1 : time_tile;
+    if (local->host_only) o.device = SDAG_DEVICE_NONE;
+    else o.device = local->device;
+    return dist_create(local->spec_text, g, o, rank, nranks, comm);
+}
+
 namespace {
 
 struct Ranges {

@@ -56,6 +56,9 @@ struct Dist {
     ~Dist();
 };
 
+// a dist from a local plan of the rank's OWNED slab (nz_own, ny, nx), every
+// rank owning nz_own planes (weak scaling): global nz = nz_own * nranks
+Dist *dist_create_local(const Plan *local, int rank, int nranks, void *comm, int time_tile);
 Dist *dist_create(const std::string &spec, const int64_t gdims[3], const sdag_plan_opts &o, int rank, int nranks,
                   void *comm);
 void dist_apply(Dist *d, double *const *a3, int n3, const double *const *a1, int n1, const double *s, int ns,

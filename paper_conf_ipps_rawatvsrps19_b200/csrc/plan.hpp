@@ -38,6 +38,8 @@ struct Plan {
     int tune = 0;
     bool tune_cached = false;  // tune=1 result restored from $SDAG_TUNE_CACHE
     std::string force_variant;
+    std::string spec_text;      // the spec this plan was created from (empty for program stages)
+    sdag_plan_opts opts_copy{};  // the options it was created with (force_variant -> the string above)
 
     // ABI mapping (per 3D formal kind_index): staged-input slot / output slot / inout slot
     std::vector<int> in_slot, out_slot, io_slot;

@@ -643,7 +643,10 @@ static bool tune_cache_load(Plan *p);
 static void tune_cache_store(const Plan *p);
 
 Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_plan_opts &o) {
-    return plan_create_from(parse_spec(spec), dims, o);  // a1
+    Plan *p = plan_create_from(parse_spec(spec), dims, o);  // a1
+    p->spec_text = spec;
+    p->opts_copy = o;
+    return p;
 }
 
 Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &o) {

@@ -186,3 +186,23 @@ def test_p2p_entry_points_fail_cleanly_without_a_device():
         assert e.value.code == code
     with pytest.raises(ValueError):
         d.p2p_attach(1, b"short")
+
+
+def test_dist_from_a_local_plan_matches_the_global_form():
+    """SURVEY 8(b)'s sdag_dist_create(local plan, ...): a plan of the owned slab
+    (nz_own, ny, nx) gives the same slab layout and local plan as the global
+    form with nz = nz_own * nranks, for every rank and ghost depth"""
+    import paper_conf_ipps_rawatvsrps19_b200 as sdag
+    for name, tt in (("smooth27", 1), ("smooth27", 2), ("lap25", 1)):
+        spec = sdag.spec_text(name)
+        local = sdag.Plan(spec, (24, 20, 22), device="none")
+        for P in (1, 2, 3):
+            for r in range(P):
+                a = sdag.Dist.from_local_plan(local, r, P, time_tile=tt)
+                b = sdag.Dist(spec, (24 * P, 20, 22), r, P, device="none", time_tile=tt)
+                assert a.layout() == b.layout(), (name, tt, P, r)
+                assert a.plan.info["variant"] == b.plan.info["variant"]
+    prog = sdag.Program(sdag.fission(sdag.spec_text("rhs4center"), "trivial"), (20, 20, 20), device="none")
+    with pytest.raises(sdag.SdagError) as e:
+        sdag.Dist.from_local_plan(prog.stage(0), 0, 2)
+    assert e.value.code == "UNSUPPORTED"
