@@ -63,7 +63,7 @@ def _check_sizes(arrays3d, arrays1d, dims, axes, batch=1, device=None, host=Fals
     """The C ABI takes raw pointers, so an undersized buffer would be read or
     written out of bounds on the device (TMA / stores) or on the host
     (cudaMemcpy): check every 3D array holds batch*nz*ny*nx elements, every 1D
-    array the extent of its axis, and (device arrays) the plan's device."""
+    array batch x the extent of its axis, and (device arrays) the plan's device."""
     n = int(batch) * int(dims[0]) * int(dims[1]) * int(dims[2])
     for q, t in enumerate(arrays3d):
         cnt = int(t.size) if host else int(t.numel())
@@ -77,8 +77,10 @@ def _check_sizes(arrays3d, arrays1d, dims, axes, batch=1, device=None, host=Fals
             if ax < 0:  # never read by the stencil
                 continue
             cnt = int(t.size) if host else int(t.numel())
-            if cnt != int(dims[ax]):
-                raise ValueError(f"1D array #{q} has {cnt} elements; its axis ({'zyx'[ax]}) has {int(dims[ax])}")
+            need = int(batch) * int(dims[ax])  # batched: [batch][len] (include/sdag.h)
+            if cnt != need:
+                raise ValueError(f"1D array #{q} has {cnt} elements; its axis ({'zyx'[ax]}) needs {need}"
+                                 + (f" ({batch} x {int(dims[ax])})" if batch > 1 else ""))
             if device is not None and not host and t.device.index != device:
                 raise ValueError(f"1D array #{q} is on {t.device}; the plan is on cuda:{device}")
 

@@ -101,9 +101,16 @@ void program_forest_tune(const std::string &text, const int64_t dims[3], const s
     *n_candidates = int(cands.size());
     *best = -1;
     double best_ms = 0.0;
-    cudaEvent_t e0, e1;
-    check_cuda(cudaEventCreate(&e0), "cudaEventCreate");
-    check_cuda(cudaEventCreate(&e1), "cudaEventCreate");
+    struct Events {  // released on every path (a candidate's plan or launch may throw)
+        cudaEvent_t e[2] = {nullptr, nullptr};
+        ~Events() {
+            for (cudaEvent_t x : e)
+                if (x) cudaEventDestroy(x);
+        }
+    } ev;
+    check_cuda(cudaEventCreate(&ev.e[0]), "cudaEventCreate");
+    check_cuda(cudaEventCreate(&ev.e[1]), "cudaEventCreate");
+    cudaEvent_t e0 = ev.e[0], e1 = ev.e[1];
     for (size_t c = 0; c < cands.size(); c++) {
         std::unique_ptr<Program> g(program_create(fuse_groups(text, cands[c]), dims, o));
         std::vector<float> t;
@@ -124,8 +131,6 @@ void program_forest_tune(const std::string &text, const int64_t dims[3], const s
             best_ms = med;
         }
     }
-    cudaEventDestroy(e0);
-    cudaEventDestroy(e1);
 }
 
 }  // namespace sdag

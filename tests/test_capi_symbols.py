@@ -91,7 +91,7 @@ def test_binding_rejects_undersized_host_buffers():
         plan.apply_host([np.zeros((8, 9, 9)), ok], scalars=[4.0, 0.5, 0.25])
     r4 = sdag.Plan(sdag.spec_text("rhs4center"), (8, 9, 10), device="none")
     g = [np.zeros((8, 9, 10)) for _ in range(8)]
-    with _pt.raises(ValueError, match="axis"):
+    with _pt.raises(ValueError, match="axis"):  # strz has the y extent
         r4.apply_host(g, [np.zeros(10), np.zeros(9), np.zeros(9)], scalars=[0.75, 1 / 6, 1 / 144, 1.0, 1.0])
 
 
