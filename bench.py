@@ -362,6 +362,7 @@ def run_reference(args):
         return 0
     import oracle
     import synth
+    world = int(os.environ.get("WORLD_SIZE", str(args.gpus)))
     ins, sc = synth.lap25_inputs((512, 512, 512), cfg="cfg2")
     A = ins["A"]
     c = [sc[k] for k in ("c0", "c1", "c2", "c3", "c4")]
@@ -377,11 +378,10 @@ def run_reference(args):
     dt = sum(times)
     pts = args.steps * 504 ** 3
     val = pts * 29 / dt / 1e9
-    world = int(os.environ.get("WORLD_SIZE", str(args.gpus)))
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "GFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": headline_config(1),
+            "config": headline_config(world),
             "cpu_baseline": {"value": val, "unit": "GFLOP/s", "cores": cpu_cores(), "kind": "oracle",
                              "cpu_model": cpu_model(), "best_step_gflops": 504 ** 3 * 29 / min(times) / 1e9,
                              "sample": f"{args.steps} full 512^3 sweeps of the benchmark input (all {504 ** 3} "
@@ -394,6 +394,11 @@ def run_reference(args):
 # ---------------------------------------------------------------------------
 # multi-GPU: config 5 as z-slabs (the BASELINE weak-scaling workload)
 # ---------------------------------------------------------------------------
+
+def _red_dev(halo):
+    """tensors for the timing reductions: the gloo group of the p2p path reduces on the host"""
+    return "cpu" if halo == "p2p" else "cuda"
+
 
 def measure_config5_slabs(tdist, rank, world, local, steps, warmup, comm, halo="nccl"):
     """Config 5 per rank: 1024^3 owned planes, T = 12, ghost depth 2 (one NCCL
@@ -440,11 +445,11 @@ def measure_config5_slabs(tdist, rank, world, local, steps, warmup, comm, halo="
         step = lambda: dd.apply_iterated(x0, x1, T, scalars=scal, stream=stream, comm_stream=cs)  # noqa: E731
     tdist.barrier()
     msN, lps, clk = timed(step, steps, warmup, stream, local)
-    t = torch.tensor([ms1, msN], dtype=torch.float64, device="cuda")
+    t = torch.tensor([ms1, msN], dtype=torch.float64, device=_red_dev(halo))
     tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
     ms1m, msNm = float(t[0]), float(t[1])
     pts = torch.tensor([float((part["k_hi"] - part["k_lo"]) * (ny - 2) * (nx - 2) * T)], dtype=torch.float64,
-                       device="cuda")
+                       device=_red_dev(halo))
     tdist.all_reduce(pts, op=tdist.ReduceOp.SUM)
     info = dd.plan.info
     del x0, step
@@ -526,16 +531,24 @@ def main():
     import synth
 
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    # SDAG_BENCH_SAME_DEVICE=1: every rank on cuda:0 (plumbing check of the N > 1
+    # code path on a one-GPU box; needs --halo p2p, NCCL refuses duplicate GPUs)
+    same = bool(os.environ.get("SDAG_BENCH_SAME_DEVICE"))
+    local = 0 if same else int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
+    p2p = args.halo == "p2p"
+    rdev = _red_dev(args.halo)
     tdist = None
     comm = None
     if world > 1:
         import torch.distributed as tdist
-        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        uid = [sdag.nccl_unique_id() if rank == 0 else None]
-        tdist.broadcast_object_list(uid, src=0)
-        comm = sdag.nccl_comm_create(uid[0], world, rank, local)
+        if p2p:  # host plumbing only: IPC handles, barriers, the timing reductions
+            tdist.init_process_group("gloo")
+        else:
+            tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+            uid = [sdag.nccl_unique_id() if rank == 0 else None]
+            tdist.broadcast_object_list(uid, src=0)
+            comm = sdag.nccl_comm_create(uid[0], world, rank, local)
     peak_hbm, peak_src = load_peaks()
     stream = torch.cuda.current_stream()
     spec = sdag.spec_text("lap25")
@@ -559,21 +572,39 @@ def main():
         dd = sdag.Dist(spec, (n * world, n, n), rank, world, comm=comm, tune=args.tune, variant=args.variant)
         (nza, ny, nx), g0 = dd.layout()
         part = sdag.slab_partition(n * world, 4, world, rank)
-        dA = synth.uniform_torch((nza, ny, nx), -1.0, 1.0, "cfg2-slab", rank)
-        dB = torch.zeros((nza, ny, nx), dtype=torch.float64, device="cuda")
+        src = synth.uniform_torch((nza, ny, nx), -1.0, 1.0, "cfg2-slab", rank)
         cs = torch.cuda.Stream()
+        if p2p:
+            # the sweep's boundary bands go to the neighbours' ghost planes by P2P
+            # (flag-ordered, CUDA IPC); one sweep = p2p_apply_iterated with T = 1
+            dA, dB = dd.p2p_alloc()
+            dA.copy_(src)
+            hs = [None] * world
+            tdist.all_gather_object(hs, dd.p2p_handle())
+            if rank > 0:
+                dd.p2p_attach(0, hs[rank - 1])
+            if rank < world - 1:
+                dd.p2p_attach(1, hs[rank + 1])
+            torch.cuda.synchronize()
+
+            def step():
+                dd.p2p_apply_iterated(1, scalars=c, stream=stream)
+        else:
+            dA = src
+            dB = torch.zeros((nza, ny, nx), dtype=torch.float64, device="cuda")
+
+            def step():
+                dd.apply([dB, dA], scalars=c, stream=stream, comm_stream=cs)
+        del src
         kplan = dd.plan
         info = kplan.info
-
-        def step():
-            dd.apply([dB, dA], scalars=c, stream=stream, comm_stream=cs)
         tdist.barrier()
         ms, lps, clk = timed(step, args.steps, args.warmup, stream, local)
-        t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+        t = torch.tensor([ms], dtype=torch.float64, device=rdev)
         tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
         ms = float(t[0])
         p = torch.tensor([float((part["k_hi"] - part["k_lo"]) * (ny - 8) * (nx - 8))], dtype=torch.float64,
-                         device="cuda")
+                         device=rdev)
         tdist.all_reduce(p, op=tdist.ReduceOp.SUM)
         pts_total = float(p[0])
         # the dominant kernel alone (same stream, same launch configuration)
@@ -619,18 +650,19 @@ def main():
                 tdist.barrier()
                 t0 = time.perf_counter()
                 dA[own].copy_(hA, non_blocking=True)
-                dd.apply([dB, dA], scalars=c, stream=stream, comm_stream=cs)
+                step()
                 hB.copy_(dB[kk], non_blocking=True)
                 stream.synchronize()
                 if it:
                     ee.append(time.perf_counter() - t0)
-            t = torch.tensor([statistics.median(ee)], dtype=torch.float64, device="cuda")
+            t = torch.tensor([statistics.median(ee)], dtype=torch.float64, device=rdev)
             tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
             te = float(t[0])
             e2e = {"value": pts_total * info["flops_per_point"] / te / 1e9, "unit": "GFLOP/s",
                    "h2d_bytes_per_step": int(hA.numel() * 8), "d2h_bytes_per_step": int(hB.numel() * 8),
                    "ms_per_step": te * 1e3, "per_rank_bytes": True,
-                   "path": "owned planes H2D + Dist.apply (NCCL halo) + computed planes D2H"}
+                   "path": "owned planes H2D + the halo-exchanged sweep (" + ("P2P stores" if p2p else "NCCL")
+                   + ") + computed planes D2H"}
     del dA, dB
     torch.cuda.empty_cache()
 
