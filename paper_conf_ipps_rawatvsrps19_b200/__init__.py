@@ -296,6 +296,8 @@ class Program:
         d = (ctypes.c_int64 * 3)(*[int(x) for x in dims])
         o = _opts(order, device, tune, batch, variant, True)
         _check(self._L.sdag_program_create(spec.encode(), d, ctypes.byref(o), ctypes.byref(self._h)))
+        self._dims = tuple(int(x) for x in dims)
+        self._device = int(o.device) if o.device >= 0 else None
 
     def close(self):
         if self._h:
@@ -346,6 +348,8 @@ class Program:
     def apply(self, arrays3d, arrays1d=(), scalars=(), stream=None, batch=1):
         p3 = [_ptr(t, "grid array") for t in arrays3d]
         p1 = [_ptr(t, "1D array") for t in arrays1d]
+        axes = [a[3] for a in self.args() if a[0] == 1]
+        _check_sizes(arrays3d, arrays1d, self._dims, axes, batch, self._device)
         s, ns = _scal(scalars)
         _check(self._L.sdag_program_apply(self._h, int(batch), _arr(p3), len(p3), _arr(p1), len(p1), s, ns,
                                           _stream_handle(stream)))
