@@ -256,9 +256,11 @@ def measure_config(cid, steps, warmup, peak_hbm, peak_src, fp64_peak, tune=False
     info = plan.info
     arrays3d, arrays1d, scal = build_arrays(sdag, plan, name, dims, batch)
     stream = torch.cuda.current_stream()
+    launch = [ln.strip() for ln in plan.describe().splitlines() if ln.strip().startswith("launch:")]
     res = {"workload": WORKLOAD[cid], "stencil": name, "grid": list(dims), "batch": batch, "sweeps_per_step": T,
            "variant": info["variant"], "flops_per_point": info["flops_per_point"],
-           "bytes_per_point": info["bytes_per_point"]}
+           "bytes_per_point": info["bytes_per_point"], "tuned": bool(tune),
+           "launch": launch[0] if launch else None}
     if cid == "1":
         # one 2 MB problem: latency-bound (launch + one short z-stream); L2 flushed
         # between iterations, each launch timed alone with events
@@ -495,7 +497,8 @@ def main():
     ap.add_argument("--no-per-config", action="store_true", help="headline only")
     ap.add_argument("--configs", default="1,1b,3,4,5", help="per_config entries at N = 1")
     ap.add_argument("--variant", default=None, help="force the headline plan's variant")
-    ap.add_argument("--tune", action="store_true", help="tune=1 plans (measured pick) instead of the heuristic")
+    ap.add_argument("--tune", action="store_true", help="headline: tune=1 plan (measured pick) instead of the heuristic")
+    ap.add_argument("--no-tune-configs", action="store_true", help="per_config: heuristic plans instead of tune=1")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--cpu-baseline-only", action="store_true", help=argparse.SUPPRESS)
     ap.add_argument("--halo", default="nccl", choices=["nccl", "p2p"], help="N > 1: config 5's slab halo path")
@@ -672,7 +675,11 @@ def main():
         if world == 1:
             fp64 = sdag.fp64_peak()
             for cid in [x for x in args.configs.split(",") if x]:
-                per[cid] = measure_config(cid, min(args.steps, 10), 3, peak_hbm, peak_src, fp64, tune=args.tune)
+                # the per-config lines use the plan-time measured pick (tune=1: hierarchical
+                # over geometries, variants and the z-chunk length), as a production user
+                # would; the headline keeps the heuristic plan unless --tune
+                per[cid] = measure_config(cid, min(args.steps, 10), 3, peak_hbm, peak_src, fp64,
+                                          tune=not args.no_tune_configs)
             per["fp64_peak_tflops_measured"] = fp64 / 1e12
         else:
             per["5"] = measure_config5_slabs(tdist, rank, world, local, min(args.steps, 5), 3, comm, args.halo)

@@ -168,6 +168,13 @@ static void geometry(const Plan *p, const KernelDesc &k, int batch, int64_t klo,
     //    unit keeps radius-4 stencils at long chunks (lap25: 8 chunks of 63).
     // z-halo planes a unit streams beyond its chunk, per side (radius x fused sweeps)
     const int64_t halo = k.tsteps > 1 ? int64_t(k.rz) * k.tsteps : int64_t(std::max(k.rz, k.rzr));
+    // weight of a unit's re-streamed z-halo planes: radius-1 kernels re-read 2
+    // planes that the neighbouring chunk's CTAs (running alongside) just pulled
+    // into L2, so they cost a fraction of a streamed plane -- measured (round 2,
+    // tools/chunk_sweep.py): batched 64^3 Jacobi best at 16-20 chunks of 3-4
+    // planes (0.1056 ms vs 0.1107 at the unweighted model's 6), while radius-4
+    // lap25 stays best at 8 chunks of 63 (its 8-plane halo is a real refill)
+    const double hw = halo <= 1 ? 0.25 : 1.0;
     double best = 1e300;
     int bestn = 1;
     const int maxn = int(std::min<int64_t>(nzi, std::max<int64_t>(1, 65535 / std::max(batch, 1))));
@@ -179,7 +186,7 @@ static void geometry(const Plan *p, const KernelDesc &k, int batch, int64_t klo,
             const double waves = double((units + slots - 1) / slots);
             cost = waves * double(zc + 2 * halo + 2);
         } else {
-            const double tu = double(zc + 2 * halo);
+            const double tu = double(zc) + 2.0 * hw * double(halo);
             cost = double(units) * tu / double(slots) + tu;
         }
         if (cost < best - 1e-9) {
@@ -819,8 +826,15 @@ Plan *plan_create_from(Stencil st, const int64_t dims[3], const sdag_plan_opts &
       << (p->tune ? (p->tune_cached ? "  [tuned, from $SDAG_TUNE_CACHE]"
                                     : "  [tuned: " + std::to_string(p->tuned_timed) + " candidates timed]")
                   : "  [heuristic]")
-      << (p->zchunk_tuned > 0 ? "  z-chunk " + std::to_string(p->zchunk_tuned) + " planes (tuned)" : "")
-      << "\n  candidates:";
+      << (p->zchunk_tuned > 0 ? "  z-chunk " + std::to_string(p->zchunk_tuned) + " planes (tuned)" : "");
+    if (!p->host_only) {  // the launch geometry of a full sweep (concurrent streaming model)
+        Launch L;
+        geometry(p.get(), k, std::max(1, p->batch_hint), p->lo[0], p->hi[0], p->lo, p->hi, L);
+        d << "\n  launch: " << L.tiles_x << " x " << L.tiles_y << " tiles x " << L.nchunk << " z-chunks of "
+          << L.zchunk << " planes" << (std::max(1, p->batch_hint) > 1 ? " x " + std::to_string(p->batch_hint) + " problems" : "")
+          << ", " << occupancy_of(p.get(), k) << " CTA(s)/SM";
+    }
+    d << "\n  candidates:";
     for (auto *c : p->cands) d << " " << c->variant;
     if (!p->fused.empty()) {
         d << "\n  temporal fusion (apply_iterated):";
