@@ -30,6 +30,11 @@ namespace dev {
 //   origin still 16-B aligned), a patch starts at an odd smem column, and its
 //   window [c-1, c+UX] is exactly UX/2 + 1 aligned pairs -- a third fewer
 //   shared-memory reads per fold for UX = 2 (the fused kernel is bound by them).
+template <bool V>
+struct BoolTag {
+    static constexpr bool value = V;
+};
+
 template <int GX, int GY, int UY, int PF, int UX = 2, bool ODD = false>
 struct Fuse2Geo {
     static constexpr int ML = ODD ? 3 : 2;       // box x margin (region - ML): 16-B alignment of the box origin
@@ -164,93 +169,116 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
     // (measured, r02, ms per sweep at 1024^3: unrolling this loop by 2 so the
     // retimed state changes roles instead of moving, 2.39 -> 2.46; skipping the
     // per-point ring select in tiles away from the global ring, -> 2.48)
-    for (int p = p0; p <= plast; p++) {
-        if (p + PF <= plast) issue(p + PF);
-        mbar_wait(&full[unsigned(p - p0) % NS], (unsigned(p - p0) / NS) & 1);
-        // ---- sweep 1: input plane p completes sweep-1 plane j = p-1 on the region ----
-        double cc[UY][UX], uu[UY][UX], s0[UY][UX];
-        fold(ring + (unsigned(p - p0) % NS) * PAL, cc, uu, s0);
-        __syncwarp();
-        if ((t & 31) == 0)
-            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[unsigned(p - p0) % NS]))
-                         : "memory");
-        const int j = p - 1;
-        const bool zring = j < a.zr_lo || j >= a.zr_hi;
-        double *s1 = s1buf + (j & 1) * PAL;
-#pragma unroll
-        for (int py = 0; py < UY; py++) {
-            double v[UX];
-#pragma unroll
-            for (int px = 0; px < UX; px++) {
-                if constexpr (FORM == 0 || FORM == 2) {
-                    v[px] = FORM == 0 ? fma(nu, T1[py][px] + uu[py][px], A1[py][px]) : T1[py][px] + uu[py][px];
-                    T1[py][px] = U1[py][px] + cc[py][px];
-                    U1[py][px] = uu[py][px];
-                } else {
-                    v[px] = ja * A1[py][px] - jc * (T1[py][px] + s0[py][px]);
-                    T1[py][px] = fma(-6.0, s0[py][px], cc[py][px] + A1[py][px]);
-                }
-                if (zring || ringxy[py][px]) v[px] = A1[py][px];  // ring: not updated by sweep 1
-                A1[py][px] = s0[py][px];
-            }
-#pragma unroll
-            for (int px = 0; px < UX; px += 2) {
-                double *q = s1 + (cy + py + 1) * PX + cx + ML + px;
-                if constexpr (ODD) {
-                    // two 8-byte stores at a 16-byte lane stride are 2-way bank
-                    // conflicted (ncu r02: 50 % excess wavefronts on these four
-                    // STS.64, 15 % of the kernel's).  Measured and reverted (r02):
-                    // aligned STS.128 pairs completed by a shuffle of the next
-                    // lane's value cut the conflicts 137 M -> 46 M per launch but
-                    // ran 4.51 -> 5.00 ms per launch: the store side is not the
-                    // bound, the fold's dependency chains are (issue 58 %).
-                    q[0] = v[px];
-                    q[1] = v[px + 1];
-                } else {
-                    *reinterpret_cast<double2 *>(q) = make_double2(v[px], v[px + 1]);
-                }
-            }
-        }
-        __syncthreads();  // sweep-1 plane j is complete in shared memory
-        if (j < kb - 1) continue;  // sweep-2 state starts at sweep-1 plane kb-1
-        // ---- sweep 2: sweep-1 plane j completes output plane k = j-1 on the tile ----
-        fold(s1, cc, uu, s0);
-        const int k = j - 1;
-        double *o = a.out[0] + ((zbase + k) * a.ny + (ry0 + cy)) * a.nx + gi;
-        const bool mp = MIR && mirror_plane(a, k);
-#pragma unroll
-        for (int py = 0; py < UY; py++) {
-            double res[UX];
-#pragma unroll
-            for (int px = 0; px < UX; px++) {
-                if constexpr (FORM == 0 || FORM == 2) {
-                    res[px] = FORM == 0 ? fma(nu, T2[py][px] + uu[py][px], A2[py][px]) : T2[py][px] + uu[py][px];
-                    T2[py][px] = U2[py][px] + cc[py][px];
-                    U2[py][px] = uu[py][px];
-                } else {
-                    res[px] = ja * A2[py][px] - jc * (T2[py][px] + s0[py][px]);
-                    T2[py][px] = fma(-6.0, s0[py][px], cc[py][px] + A2[py][px]);
-                }
-                A2[py][px] = s0[py][px];
-            }
-            const int ry = cy + py, gj = ry0 + ry;
-            if (k >= kb && ry >= 1 && ry <= TY && gj < a.hi[1]) {
-#pragma unroll
-                for (int px = 0; px < UX; px += 2) {
-                    if (vec_ok && outm[px] && outm[px + 1]) {
-                        __stcs(reinterpret_cast<double2 *>(o + px), make_double2(res[px], res[px + 1]));
-                        if constexpr (MIR) if (mp) mirror2(a, k, o + px, res[px], res[px + 1]);
+    // the plane loop, compiled twice: CTAs whose region touches the global x/y
+    // ring keep the per-point ring select of sweep 1, all others have none
+    // (ncu r02: the select and its recomputed predicates were ~4 instructions
+    // per point-sweep of 45)
+    auto run = [&](auto ring_tag) {
+        constexpr bool RING = decltype(ring_tag)::value;
+        for (int p = p0; p <= plast; p++) {
+            if (p + PF <= plast) issue(p + PF);
+            mbar_wait(&full[unsigned(p - p0) % NS], (unsigned(p - p0) / NS) & 1);
+            // ---- sweep 1: input plane p completes sweep-1 plane j = p-1 on the region ----
+            double cc[UY][UX], uu[UY][UX], s0[UY][UX];
+            fold(ring + (unsigned(p - p0) % NS) * PAL, cc, uu, s0);
+            __syncwarp();
+            if ((t & 31) == 0)
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&empty[unsigned(p - p0) % NS]))
+                             : "memory");
+            const int j = p - 1;
+            const bool zring = j < a.zr_lo || j >= a.zr_hi;
+            double *s1 = s1buf + (j & 1) * PAL;
+            double v[UY][UX], keep[UY][UX];
+    #pragma unroll
+            for (int py = 0; py < UY; py++)
+    #pragma unroll
+                for (int px = 0; px < UX; px++) {
+                    keep[py][px] = A1[py][px];  // the input value: what a ring point keeps
+                    if constexpr (FORM == 0 || FORM == 2) {
+                        v[py][px] = FORM == 0 ? fma(nu, T1[py][px] + uu[py][px], A1[py][px]) : T1[py][px] + uu[py][px];
+                        T1[py][px] = U1[py][px] + cc[py][px];
+                        U1[py][px] = uu[py][px];
                     } else {
-                        if (outm[px]) __stcs(o + px, res[px]);
-                        if (outm[px + 1]) __stcs(o + px + 1, res[px + 1]);
-                        if (MIR && mp && outm[px]) mirror1(a, k, o + px, res[px]);
-                        if (MIR && mp && outm[px + 1]) mirror1(a, k, o + px + 1, res[px + 1]);
+                        v[py][px] = ja * A1[py][px] - jc * (T1[py][px] + s0[py][px]);
+                        T1[py][px] = fma(-6.0, s0[py][px], cc[py][px] + A1[py][px]);
+                    }
+                    if constexpr (RING)
+                        if (ringxy[py][px]) v[py][px] = keep[py][px];  // x/y ring: not updated by sweep 1
+                    A1[py][px] = s0[py][px];
+                }
+            // the sweep-1 plane into shared memory; a global z-ring plane keeps its
+            // input (a CTA-uniform branch between two store sequences, no per-point select)
+            auto store = [&](const double(&w)[UY][UX]) {
+    #pragma unroll
+                for (int py = 0; py < UY; py++)
+    #pragma unroll
+                    for (int px = 0; px < UX; px += 2) {
+                        double *q = s1 + (cy + py + 1) * PX + cx + ML + px;
+                        if constexpr (ODD) {
+                            // two 8-byte stores at a 16-byte lane stride are 2-way bank
+                            // conflicted (ncu r02: 50 % excess wavefronts on these four
+                            // STS.64, 15 % of the kernel's).  Measured and reverted (r02):
+                            // aligned STS.128 pairs completed by a shuffle of the next
+                            // lane's value cut the conflicts 137 M -> 46 M per launch but
+                            // ran 4.51 -> 5.00 ms per launch: the store side is not the
+                            // bound, the fold's dependency chains are (issue 58 %).
+                            q[0] = w[py][px];
+                            q[1] = w[py][px + 1];
+                        } else {
+                            *reinterpret_cast<double2 *>(q) = make_double2(w[py][px], w[py][px + 1]);
+                        }
+                    }
+            };
+            if (zring)
+                store(keep);
+            else
+                store(v);
+            __syncthreads();  // sweep-1 plane j is complete in shared memory
+            if (j < kb - 1) continue;  // sweep-2 state starts at sweep-1 plane kb-1
+            // ---- sweep 2: sweep-1 plane j completes output plane k = j-1 on the tile ----
+            fold(s1, cc, uu, s0);
+            const int k = j - 1;
+            double *o = a.out[0] + ((zbase + k) * a.ny + (ry0 + cy)) * a.nx + gi;
+            const bool mp = MIR && mirror_plane(a, k);
+    #pragma unroll
+            for (int py = 0; py < UY; py++) {
+                double res[UX];
+    #pragma unroll
+                for (int px = 0; px < UX; px++) {
+                    if constexpr (FORM == 0 || FORM == 2) {
+                        res[px] = FORM == 0 ? fma(nu, T2[py][px] + uu[py][px], A2[py][px]) : T2[py][px] + uu[py][px];
+                        T2[py][px] = U2[py][px] + cc[py][px];
+                        U2[py][px] = uu[py][px];
+                    } else {
+                        res[px] = ja * A2[py][px] - jc * (T2[py][px] + s0[py][px]);
+                        T2[py][px] = fma(-6.0, s0[py][px], cc[py][px] + A2[py][px]);
+                    }
+                    A2[py][px] = s0[py][px];
+                }
+                const int ry = cy + py, gj = ry0 + ry;
+                if (k >= kb && ry >= 1 && ry <= TY && gj < a.hi[1]) {
+    #pragma unroll
+                    for (int px = 0; px < UX; px += 2) {
+                        if (vec_ok && outm[px] && outm[px + 1]) {
+                            __stcs(reinterpret_cast<double2 *>(o + px), make_double2(res[px], res[px + 1]));
+                            if constexpr (MIR) if (mp) mirror2(a, k, o + px, res[px], res[px + 1]);
+                        } else {
+                            if (outm[px]) __stcs(o + px, res[px]);
+                            if (outm[px + 1]) __stcs(o + px + 1, res[px + 1]);
+                            if (MIR && mp && outm[px]) mirror1(a, k, o + px, res[px]);
+                            if (MIR && mp && outm[px + 1]) mirror1(a, k, o + px + 1, res[px + 1]);
+                        }
                     }
                 }
+                o += a.nx;
             }
-            o += a.nx;
         }
-    }
+    };
+    const bool tile_ring = ry0 <= 0 || ry0 + GY - 1 >= ny - 1 || rx0 <= 0 || rx0 + GX - 1 >= nx - 1;
+    if (tile_ring)
+        run(BoolTag<true>{});
+    else
+        run(BoolTag<false>{});
 }
 
 }  // namespace dev
