@@ -175,6 +175,7 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
     // per point-sweep of 45)
     auto run = [&](auto ring_tag) {
         constexpr bool RING = decltype(ring_tag)::value;
+#pragma unroll 2
         for (int p = p0; p <= plast; p++) {
             if (p + PF <= plast) issue(p + PF);
             mbar_wait(&full[unsigned(p - p0) % NS], (unsigned(p - p0) / NS) & 1);
