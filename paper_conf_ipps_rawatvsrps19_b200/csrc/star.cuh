@@ -202,8 +202,9 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
     // queue slot of plane k + d (k = p - R) when plane p sits in slot PH
     auto qs = [](int ph, int d) { return ROT ? (ph + NQ - R + d) % NQ : ph - R + d; };
 
-    auto step = [&](auto phase, int p) {
+    auto step = [&](auto phase, int p, auto full_tag) {
         constexpr int PH = decltype(phase)::value;  // slot of plane p in q
+        constexpr bool FULL = decltype(full_tag)::value;  // every output of this CTA is interior
         {
             const int pn = p + PF;
             if (pn <= plast) issue(pn);
@@ -388,6 +389,16 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
             // interior-only streaming stores (16-B vector stores when both points are inside)
             double *o = a.out[0] + ((zbase + k) * a.ny + (y0 + cy)) * a.nx + gi;
             const bool mp = MIR && mirror_plane(a, k);  // dist p2p: also into a neighbour's ghosts
+            if constexpr (FULL && QMODE != 3) {
+                // a tile entirely inside the interior (the common case): 16-B
+                // stores with no per-row / per-point conditions
+#pragma unroll
+                for (int py = 0; py < UY; py++) {
+                    __stcs(reinterpret_cast<double2 *>(o), make_double2(acc[py][0], acc[py][1]));
+                    if constexpr (MIR) if (mp) mirror2(a, k, o, acc[py][0], acc[py][1]);
+                    o += a.nx;
+                }
+            } else {
 #pragma unroll
             for (int py = 0; py < UY; py++) {
                 // QMODE 3 (code differencing): arithmetic kept alive, stores (almost) never issued
@@ -404,22 +415,27 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
                 }
                 o += a.nx;
             }
+            }
         } else if (p < kb) {
             release(p);  // a head-only plane (never a centre) is done
         }
         if constexpr (!USE_TMA) __syncthreads();  // the LSU ring has no empty barriers
     };
 
+    // the plane loop, compiled twice: tiles whose outputs are all interior (and
+    // 16-B aligned) store without per-row / per-point conditions
+    auto run = [&](auto full_tag) {
     if constexpr (QMODE == 6) {
         for (int p = p0; p <= plast; p += NQ)
             static_for<NQ>([&](auto I) {
-                if (p + decltype(I)::value <= plast) step(I, p + decltype(I)::value);
+                if (p + decltype(I)::value <= plast) step(I, p + decltype(I)::value, full_tag);
             });
     } else if constexpr (QMODE != 1) {
         for (int p = p0; p <= plast; p += UNR) {
             static_for<UNR>([&](auto I) {
                 if (UNR == 1 || p + decltype(I)::value <= plast)
-                    step(std::integral_constant<int, NQ - 1 + decltype(I)::value>{}, p + decltype(I)::value);
+                    step(std::integral_constant<int, NQ - 1 + decltype(I)::value>{}, p + decltype(I)::value,
+                         full_tag);
             });
 #pragma unroll
             for (int d = 0; d < NQ - 1; d++)
@@ -433,10 +449,17 @@ __global__ void __launch_bounds__(StarGeo<B, TX, TY, UY, PF>::THREADS, MINB)
         for (int p = p0; p <= plast; p++) {
             const int ph = unsigned(p - p0) % NQ;
             static_for<NQ>([&](auto I) {
-                if (ph == decltype(I)::value) step(I, p);
+                if (ph == decltype(I)::value) step(I, p, full_tag);
             });
         }
     }
+    };
+    const bool tile_full = x0 >= a.xmin && x0 + TX <= a.hi[2] && y0 + TY <= a.hi[1] && (a.nx % 2 == 0) &&
+                      ((reinterpret_cast<uintptr_t>(a.out[0]) & 15) == 0);
+    if (tile_full)
+        run(std::integral_constant<bool, true>{});
+    else
+        run(std::integral_constant<bool, false>{});
 }
 
 
