@@ -7,6 +7,9 @@ void add_kernels_hypterm(std::vector<KernelDesc> &v) {
     SDAG_HYP_PAIR(v, "hypterm", 64, 8, 2, 0);  // 0.793-0.796 ms at 320^3 (pf1: 0.826)
     // cropped per-array boxes: 0.799 ms (32x16: 0.874), no gain -- DESIGN 6.4
     SDAG_HYPC_PAIR(v, "hypterm", 64, 8, 2, 1);
+    // round 2, measured and removed: thread 0 issuing TMA without blocking on the
+    // slot (mbarrier.test_wait at three points of the plane, blocking only for the
+    // plane needed next) 0.876 ms (pf2) / 0.873 (pf1) vs 0.794 -- DESIGN 6.4
     SDAG_HYP_PAIR(v, "hypterm", 16, 16, 2, 1);
     SDAG_HYP_PAIR(v, "hypterm", 64, 8, 1, 2);
     SDAG_HYP_PAIR(v, "hypterm", 32, 16, 1, 3);
