@@ -236,7 +236,9 @@ __global__ void __launch_bounds__(Fuse2Geo<GX, GY, UY, PF, UX, ODD>::THREADS, MI
                 store(v);
             // (measured, r02: handing the plane from row block to row block with
             // per-warp counters -- lane-0 spin on ld.acquire, st.release -- instead
-            // of this barrier ran 2.2 -> 4.1 ms per sweep)
+            // of this barrier ran 2.2 -> 4.1 ms per sweep; running sweep 2 one plane
+            // behind through four slots and per-slot mbarriers (hardware-suspended
+            // waits, no CTA barrier) 2.22 -> 2.45)
             __syncthreads();  // sweep-1 plane j is complete in shared memory
             if (j < kb - 1) continue;  // sweep-2 state starts at sweep-1 plane kb-1
             // ---- sweep 2: sweep-1 plane j completes output plane k = j-1 on the tile ----
