@@ -134,6 +134,10 @@ __global__ void __launch_bounds__(HypGeo<TX, TY, PF>::THREADS, 1)
 #pragma unroll
         for (int m = 0; m < 5; m++) acc[j][m][0] = acc[j][m][1] = 0.0;
 
+    // the plane loop, compiled twice: tiles entirely inside the interior (16-B
+    // aligned outputs) store without per-row / per-point conditions
+    auto run = [&](auto full_tag) {
+    constexpr bool FULL = decltype(full_tag)::value;
     for (int p = p0; p <= plast; p++) {
         {
             const int pn = p + PF;
@@ -174,12 +178,12 @@ __global__ void __launch_bounds__(HypGeo<TX, TY, PF>::THREADS, 1)
                 }
             // ---- output p-4 is complete ----
             const int k = p - R;
-            if (k >= kb && rowok) {
+            if (k >= kb && (FULL || rowok)) {
                 const int64_t off = ((zbase + k) * a.ny + gj) * a.nx + gi;
 #pragma unroll
                 for (int m = 0; m < 5; m++) {
                     double *o = a.out[m] + off;
-                    if (vec && (reinterpret_cast<uintptr_t>(a.out[m]) & 15) == 0) {
+                    if (FULL || (vec && (reinterpret_cast<uintptr_t>(a.out[m]) & 15) == 0)) {
                         __stcs(reinterpret_cast<double2 *>(o), make_double2(acc[0][m][0], acc[0][m][1]));
                     } else {
                         if (ok0) __stcs(o, acc[0][m][0]);
@@ -268,6 +272,14 @@ __global__ void __launch_bounds__(HypGeo<TX, TY, PF>::THREADS, 1)
         }
         if constexpr (!USE_TMA) __syncthreads();
     }
+    };
+    bool tile_full = x0 >= a.xmin && x0 + TX <= a.hi[2] && y0 + TY <= a.hi[1] && (a.nx % 2 == 0);
+#pragma unroll
+    for (int m = 0; m < 5; m++) tile_full = tile_full && (reinterpret_cast<uintptr_t>(a.out[m]) & 15) == 0;
+    if (tile_full)
+        run(std::integral_constant<bool, true>{});
+    else
+        run(std::integral_constant<bool, false>{});
 }
 
 // ---------------------------------------------------------------------------
