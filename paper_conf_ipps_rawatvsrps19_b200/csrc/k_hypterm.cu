@@ -13,6 +13,8 @@ void add_kernels_hypterm(std::vector<KernelDesc> &v) {
     SDAG_HYP_PAIR(v, "hypterm", 16, 16, 2, 1);
     SDAG_HYP_PAIR(v, "hypterm", 64, 8, 1, 2);
     SDAG_HYP_PAIR(v, "hypterm", 32, 16, 1, 3);
+    // round 2, measured and removed (ms at 320^3 vs 0.779 for 64x8 pf2): 32x16 pf2
+    // 0.850 (less y-halo fill, fewer warps/SM), 32x8 pf3 1.046
     SDAG_HYP_PAIR(v, "hypterm", 32, 8, 2, 4);
     SDAG_PAIR(v, Hypterm, "hypterm", 32, 8, 1, 1, 2, 10);
 }
