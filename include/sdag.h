@@ -40,6 +40,13 @@
  *    (except sdag_apply_host, which is synchronous).  Device faults surface
  *    at the caller's next synchronisation.
  *  - No CPU fallback: a device that is not sm_100 returns SDAG_ERR_DEVICE.
+ *  - Tracing: every enqueueing entry point opens an NVTX range named after
+ *    the call ("sdag_apply <stencil> <variant>", "sdag_apply_iterated ... T=",
+ *    "sdag_dist_apply*", "sdag_halo_exchange_nccl", "sdag_program_apply",
+ *    "sdag_plan_create"), visible to nsys / ncu --nvtx.
+ *  - Environment: SDAG_LOG=1 prints each plan's sdag_plan_describe() text
+ *    (and each program stage's) to stderr at creation; SDAG_TUNE_CACHE,
+ *    SDAG_GRAPHS and SDAG_NCCL_CHECK are described where they act.
  */
 #ifndef SDAG_H
 #define SDAG_H

@@ -270,6 +270,7 @@ void exchange_nccl(Dist *d, double *const *a3, cudaStream_t comm, int planes) {
     const size_t cnt = plane * size_t(planes);
     const Halo h = halo_schedule(d->slab, planes);
     auto c = static_cast<ncclComm_t>(d->comm);
+    NvtxRange nr("sdag_halo_exchange_nccl");
     // every call between GroupStart and GroupEnd is made even after a failure,
     // and GroupEnd always runs: an open group would corrupt every later call on
     // the communicator.  The first error is reported after the group is closed.
@@ -390,6 +391,7 @@ void dist_apply(Dist *d, double *const *a3, int n3, const double *const *a1, int
         for (int f = 0; f < n3; f++)
             if (reinterpret_cast<uintptr_t>(a3[f]) % 16) throw Error(SDAG_ERR_INVALID_ARG, "grid arrays must be 16-B aligned");
     DeviceGuard dg(p);  // libsdag's runtime: bind the plan's device, restore the caller's
+    NvtxRange nr("sdag_dist_apply " + p->st.name);
     sweep_split(d, p->kernel(), a3, a1, s, compute, comm_stream(d, comm), true);
 }
 
@@ -404,6 +406,7 @@ void dist_apply_iterated(Dist *d, double *b0, double *b1, int T, const double *s
     int fin = -1, fout = -1;
     for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
     DeviceGuard dg(p);
+    NvtxRange nr("sdag_dist_apply_iterated " + p->st.name + " T=" + std::to_string(T));
     cudaStream_t cs = comm_stream(d, comm);
     double *bufs[2] = {b0, b1};
     int cur = 0;
@@ -419,6 +422,7 @@ void dist_apply_iterated(Dist *d, double *b0, double *b1, int T, const double *s
 void dist_apply_iterated_loopback(Dist **ds, int n, double *const *b0, double *const *b1, int T, const double *s,
                                   int ns, cudaStream_t stream) {
     if (!ds || n < 1) throw Error(SDAG_ERR_INVALID_ARG, "bad dist list");
+    NvtxRange nr("sdag_dist_apply_iterated_loopback T=" + std::to_string(T));
     for (int r = 0; r < n; r++) {
         if (!ds[r] || ds[r]->rank != r || ds[r]->nranks != n) throw Error(SDAG_ERR_INVALID_ARG, "dists must be ranks 0..n-1");
         if (ds[r]->local->host_only) throw Error(SDAG_ERR_DEVICE, "host-only dist plan");
@@ -597,6 +601,7 @@ void dist_p2p_apply_iterated(Dist *d, int T, const double *s, int ns, cudaStream
     for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
     DeviceGuard dg(p);
     if (T == 0) return;
+    NvtxRange nr("sdag_dist_p2p_apply_iterated " + p->st.name + " T=" + std::to_string(T));
 
     const int64_t H = S.halo;
     const size_t plane = size_t(p->dims[1] * p->dims[2]);

@@ -11,6 +11,8 @@
 #include <tuple>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "ir.hpp"
 #include "kernels.hpp"
 #include "registry.hpp"
@@ -162,6 +164,19 @@ struct DeviceGuard {
         if (prev >= 0) cudaSetDevice(prev);
     }
 };
+// NVTX range around a host entry point (tracing): the range
+// appears on the CPU timeline of nsys / ncu --nvtx so a trace names which
+// sdag call enqueued which kernels.  nvtx3 is header-only; with no tool
+// attached a push/pop is a null-pointer check.
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    explicit NvtxRange(const std::string &name) { nvtxRangePushA(name.c_str()); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange &) = delete;
+    NvtxRange &operator=(const NvtxRange &) = delete;
+};
+bool log_enabled();
+void log_plan(const Plan *p, const char *what);
 // jit.cu (NEXT-4)
 std::string jit_body_source(const Plan &p, const std::string &sname, int rzr);
 void jit_build_candidates(Plan *p);

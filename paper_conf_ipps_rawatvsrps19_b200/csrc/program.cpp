@@ -37,6 +37,7 @@ Program *program_create(const std::string &spec, const int64_t dims[3], const sd
     for (size_t s = 0; s < g->ir.stages.size(); s++) {
         g->stages.emplace_back(plan_create_from(g->ir.stages[s], dims, o));
         g->handles.push_back(new sdag_plan_s{g->stages.back().get()});
+        log_plan(g->stages.back().get(), ("program stage " + std::to_string(s)).c_str());
     }
     // program-level roles of the 3D arrays, in call order: read before any
     // stage wrote it -> In (InOut once written later); first touched by a
@@ -63,6 +64,7 @@ void program_apply(Program *g, double *const *a3, int n3, const double *const *a
                                               std::to_string(g->n_of(ArgKind::Array1D)) + " 1D arrays and " +
                                               std::to_string(g->n_of(ArgKind::Scalar)) + " scalars");
     if ((n3 && !a3) || (n1 && !a1) || (ns && !s)) throw Error(SDAG_ERR_INVALID_ARG, "null argument array");
+    NvtxRange nr("sdag_program_apply " + std::to_string(g->stages.size()) + " stages");
     // bind every stage first (all validation before anything is enqueued)
     struct Bound {
         std::vector<double *> a3;

@@ -12,6 +12,7 @@
 #include <array>
 #include <atomic>
 #include <cmath>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <memory>
@@ -379,6 +380,7 @@ void apply(Plan *p, double *const *a3, int n3, const double *const *a1, int n1, 
     if (ns > 0 && !s) throw Error(SDAG_ERR_INVALID_ARG, "null scalars");
     DeviceGuard g(p);
     const KernelDesc &k = pick_kernel(p, a3, p->dims[2]);
+    NvtxRange r("sdag_apply " + p->st.name + " " + k.variant);
     plan_launch(p, k, a3, a1, s, batch, 0, p->dims[0], stream);
 }
 
@@ -418,6 +420,7 @@ void apply_iterated(Plan *p, double *b0, double *b1, int T, const double *s, int
         throw Error(SDAG_ERR_INVALID_ARG, "apply_iterated needs a 1-input 1-output plan without 1D arrays");
     if (T < 0) throw Error(SDAG_ERR_INVALID_ARG, "T must be >= 0");
     if (!b0 || !b1 || b0 == b1) throw Error(SDAG_ERR_INVALID_ARG, "two distinct buffers required");
+    NvtxRange nr("sdag_apply_iterated " + p->st.name + " T=" + std::to_string(T));
     int fin = -1, fout = -1;
     for (int f = 0; f < 2; f++) (p->st.formal(ArgKind::Array3D, f).role == Role::In ? fin : fout) = f;
     double *bufs[2] = {b0, b1};
@@ -649,10 +652,31 @@ static void time_candidates(Plan *p);
 static bool tune_cache_load(Plan *p);
 static void tune_cache_store(const Plan *p);
 
+// SDAG_LOG=1: every plan prints its describe() text (DAG, analysis, the
+// chosen kernel, launch geometry, tuning result) to stderr when created, so
+// a run's log records which sm_100a variant served each stencil.
+bool log_enabled() {
+    static const bool on = [] {
+        const char *e = std::getenv("SDAG_LOG");
+        return e && e[0] && e[0] != '0';
+    }();
+    return on;
+}
+
+void log_plan(const Plan *p, const char *what) {
+    if (!log_enabled()) return;
+    const std::string dev = p->host_only ? std::string("none") : std::to_string(p->device);
+    std::fprintf(stderr, "[sdag] %s %s dims=(%lld,%lld,%lld) device=%s\n%s\n", what, p->st.name.c_str(),
+                 (long long)p->dims[0], (long long)p->dims[1], (long long)p->dims[2], dev.c_str(),
+                 p->describe_text.c_str());
+}
+
 Plan *plan_create(const std::string &spec, const int64_t dims[3], const sdag_plan_opts &o) {
+    NvtxRange r("sdag_plan_create");
     Plan *p = plan_create_from(parse_spec(spec), dims, o);  // a1
     p->spec_text = spec;
     p->opts_copy = o;
+    log_plan(p, "plan");
     return p;
 }
 
