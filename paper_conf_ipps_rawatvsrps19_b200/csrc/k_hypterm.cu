@@ -16,6 +16,10 @@ void add_kernels_hypterm(std::vector<KernelDesc> &v) {
     // round 2, measured and removed (ms at 320^3 vs 0.779 for 64x8 pf2): 32x16 pf2
     // 0.850 (less y-halo fill, fewer warps/SM), 32x8 pf3 1.046
     SDAG_HYP_PAIR(v, "hypterm", 32, 8, 2, 4);
+    // round 2, measured and removed: plane loop unrolled 2 / 4 / 8 (the 8-slot
+    // output ring rotated by register renaming instead of ~90 moves per plane):
+    // 0.781-0.787 / 1.27 (spills) / 1.40 (spills) ms vs 0.778 -- the moves are
+    // not on the critical path (DESIGN 6.4)
     SDAG_PAIR(v, Hypterm, "hypterm", 32, 8, 1, 1, 2, 10);
 }
 }  // namespace sdag

@@ -12,6 +12,7 @@ timeout 300 python -c "import __graft_entry__ as g; g.smoke(); print('smoke ok')
 timeout 900 python bench.py > $M/bench.json 2> $M/bench.err
 timeout 900 python bench.py --impl reference --steps 5 --warmup 3 > $M/bench_reference.json 2> $M/bench_reference.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $M/bench_launches.csv python bench.py --steps 5 --warmup 3 --no-cpu --no-e2e > /dev/null 2> $M/ncu_launches.err
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $M/bench_launches_headline.csv python bench.py --steps 5 --warmup 3 --no-cpu --no-e2e --no-per-config > /dev/null 2> $M/ncu_launches_headline.err
 FP64=smsp__sass_thread_inst_executed_op_dfma_pred_on.sum,smsp__sass_thread_inst_executed_op_dadd_pred_on.sum,smsp__sass_thread_inst_executed_op_dmul_pred_on.sum
 for d in lap25 jacobi7 hypterm rhs4center smooth27; do
   timeout 900 ncu --set full --metrics $FP64 --import-source on --clock-control none -k regex:sdag_ -c 1 -o $M/prof_$d python tools/prof_one.py $d - 2 > $M/ncu_$d.log 2>&1
