@@ -19,6 +19,10 @@ void add_kernels_lap25(std::vector<KernelDesc> &v) {
     SDAG_STAR2_PAIR(v, Lap25Star, "lap25", 32, 32, 4, 3, 1, 40);
     SDAG_STAR_LATE(v, Lap25Star, "lap25", 32, 32, 4, 3, 1, 2, 41);
     SDAG_STAR_SPLIT(v, Lap25Star, "lap25", 32, 32, 4, 3, 1, 2, 42);
+    // round 2, measured and removed (ms at 512^3, two runs): prefetch depth of the
+    // default unroll-2 kernel pf2 0.420, pf4 0.3945-0.3963 (= pf3's 0.3947-0.3950),
+    // pf5 / pf6 0.559-0.563 (the 10-11 slot ring leaves room for one CTA per SM),
+    // pf4 with unroll 3 0.399 -- the ring is deep enough at pf3 (DESIGN 6.4)
     // code differencing, profiling only: never chosen unless forced
     SDAG_STAR_DIFF(v, Lap25Star, "lap25", 32, 32, 4, 3, 2, 1000);
     SDAG_STAR_DIFF(v, Lap25Star, "lap25", 32, 32, 4, 3, 3, 1001);
