@@ -11,6 +11,9 @@ void add_kernels_rhs4(std::vector<KernelDesc> &v) {
     SDAG_RHS4F_PAIR(v, "rhs4center", 32, 16, 1, -3);
     SDAG_RHS4F_PAIR(v, "rhs4center", 32, 8, 1, -2);
     SDAG_RHS4G_PAIR(v, "rhs4center", 32, 16, -1);  // double-buffered fields, one barrier per plane
+    // round 2, measured and removed: the r4g CTA barrier split into mbarriers
+    // ("fields stored" / "fields read", warps skew by up to a phase) 1.488 ms vs
+    // 1.437 -- lock-step phases are not what holds the field kernels back (DESIGN 6.4)
     SDAG_RHS4_PAIR(v, "rhs4center", 16, 16, 1, 1, -9);
     SDAG_RHS4_PAIR(v, "rhs4center", 64, 8, 1, 1, -8);
     SDAG_RHS4_PAIR(v, "rhs4center", 32, 8, 1, 1, -7);

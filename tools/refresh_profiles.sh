@@ -25,4 +25,5 @@ for d in lap25 jacobi7 hypterm rhs4center smooth27 fuse2; do
   python3 tools/ncu_summary.py $M/prof_$d.ncu-rep $P/ncu/${d}_ncu --variant "${KEY[$d]}" > /dev/null
 done
 python3 tools/sass_evidence.py $P/sass_evidence.md
+python3 tools/floors.py $M $P/floors > /dev/null
 echo "refreshed $P"
