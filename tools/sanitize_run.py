@@ -4,7 +4,7 @@
 the P2P flag protocol).  Small grids keep the instrumented run short.
 
 usage: compute-sanitizer --tool TOOL python tools/sanitize_run.py [FAMILY ...]
-families: star box27 fuse2 fuseN hyp hypc rhs4 sweep lsu jit p2p
+families: star box27 fuse2 fuseN hyp hypc rhs4 rhs4f sweep lsu jit p2p
 """
 import sys
 from pathlib import Path
@@ -66,6 +66,7 @@ FAM = {
     "hyp": lambda: one("hypterm", (12, 20, 72)),
     "hypc": lambda: one("hypterm", (12, 20, 72), "hypc_tma_64x8_u2x1_pf2"),
     "rhs4": lambda: one("rhs4center", (9, 20, 36)),
+    "rhs4f": lambda: [one("rhs4center", (9, 20, 36), v) for v in ("r4f_tma_32x16_u2x1_pf1", "r4g_tma_32x16_u2x1_pf0")],
     "sweep": lambda: one("lap25", (12, 20, 72), "tma_64x16_u1x4_pf1"),
     "lsu": lambda: [one(n, (11, 13, 35)) for n in ("lap25", "smooth27", "hypterm", "rhs4center", "jacobi7")],
     "jit": lambda: one("lap25", (12, 20, 40), "jit"),
