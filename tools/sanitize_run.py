@@ -22,7 +22,7 @@ SCAL = {"lap25": list(synth.LAP25_COEFS.values()), "jacobi7": [4.0, 0.5, 0.25],
         "rhs4center": [0.75, 1 / 6, 1 / 144, 1.0, 1.0]}
 
 
-def one(name, dims, variant=None, iterated=0):
+def one(name, dims, variant=None, iterated=0, deg=2):
     plan = sdag.Plan(sdag.spec_text(name), dims, variant=variant)
     info = plan.info
     g = torch.Generator(device="cuda").manual_seed(3)
@@ -33,7 +33,11 @@ def one(name, dims, variant=None, iterated=0):
     else:
         plan.apply(arrs, a1, SCAL[name])
     torch.cuda.synchronize()
-    print(f"{name} {info['variant']} {plan.kernel_name(1) if not iterated else ''} ok", flush=True)
+    if iterated:  # the fused kernel apply_iterated launched (temporal fusion of `iterated` sweeps)
+        fl = [ln.strip() for ln in plan.describe().splitlines() if "temporal fusion" in ln]
+        print(f"{name} {fl[0] if fl else info['variant']} | {plan.kernel_name(deg)} ok", flush=True)
+    else:
+        print(f"{name} {info['variant']} {plan.kernel_name(1)} ok", flush=True)
 
 
 def p2p():
@@ -62,7 +66,7 @@ FAM = {
     "star": lambda: one("lap25", (20, 40, 72)),
     "box27": lambda: one("smooth27", (12, 34, 140)),
     "fuse2": lambda: one("smooth27", (12, 34, 140), "fuse2o_tma_62x14_u2x2_pf2_mb2", iterated=4),
-    "fuseN": lambda: one("smooth27", (12, 34, 140), "fuse3_tma_60x28_u2x2_pf2_mb1", iterated=3),
+    "fuseN": lambda: one("smooth27", (12, 34, 140), "fuse3_tma_60x28_u2x2_pf2_mb1", iterated=3, deg=3),
     "hyp": lambda: one("hypterm", (12, 20, 72)),
     "hypc": lambda: one("hypterm", (12, 20, 72), "hypc_tma_64x8_u2x1_pf2"),
     "rhs4": lambda: one("rhs4center", (9, 20, 36)),
