@@ -22,7 +22,9 @@ void add_kernels_lap25(std::vector<KernelDesc> &v) {
     // round 2, measured and removed (ms at 512^3, two runs): prefetch depth of the
     // default unroll-2 kernel pf2 0.420, pf4 0.3945-0.3963 (= pf3's 0.3947-0.3950),
     // pf5 / pf6 0.559-0.563 (the 10-11 slot ring leaves room for one CTA per SM),
-    // pf4 with unroll 3 0.399 -- the ring is deep enough at pf3 (DESIGN 6.4)
+    // pf4 with unroll 3 0.399 -- the ring is deep enough at pf3 (DESIGN 6.4);
+    // tile shapes with unroll 2 (less halo fill per point): 64x32 0.404, 32x64
+    // 0.401, 64x16 0.397, 32x48 0.481 (6 warps/SM) vs 32x32's 0.3944
     // code differencing, profiling only: never chosen unless forced
     SDAG_STAR_DIFF(v, Lap25Star, "lap25", 32, 32, 4, 3, 2, 1000);
     SDAG_STAR_DIFF(v, Lap25Star, "lap25", 32, 32, 4, 3, 3, 1001);
