@@ -7,6 +7,12 @@ void add_kernels_rhs4(std::vector<KernelDesc> &v) {
     // specialised kernel (rhs4.cuh): 2 x UY patches from 128-bit pair loads, derivative fields
     // (2 x 2 / 2 x 4 patches spill at 255 registers and run 3x slower; not registered)
     SDAG_RHS4_PAIR(v, "rhs4center", 32, 16, 1, 1, -10);
+    // round 2, measured and removed: two output planes per step sharing the z-tap
+    // loads of planes k-2..k+3 (7-plane ring, 226 KB of smem): correct (bitwise on
+    // the exact cases) but 1.264-1.276 ms -- ncu: 67.6 LDS.128 per point (the
+    // compiler re-loads what the per-plane order was meant to share, at 254
+    // registers) and ~50 SYNCS + 49 YIELD per point spinning on the 2-plane refill
+    // (DESIGN 6.4)
     // cooperative derivative fields + retimed z (rhs4f.cuh)
     SDAG_RHS4F_PAIR(v, "rhs4center", 32, 16, 1, -3);
     SDAG_RHS4F_PAIR(v, "rhs4center", 32, 8, 1, -2);
