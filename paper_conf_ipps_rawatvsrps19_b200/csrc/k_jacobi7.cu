@@ -3,13 +3,18 @@
 #include "kdesc.cuh"
 namespace sdag {
 void add_kernels_jacobi7(std::vector<KernelDesc> &v) {
-    SDAG_STAR_PAIR(v, Jacobi7Star, "jacobi7", 64, 16, 2, 3, 0);
+    // prefetch depth 6 (8-slot ring, 2 CTAs/SM) ahead of depth 3 (3 CTAs/SM):
+    // batched 128 x 64^3 0.1058-0.1061 ms vs 0.1072-0.1078 (round 2, two runs
+    // each); one 64^3 problem unchanged (~9 us, latency).  Measured and not
+    // registered: pf3/pf4 at 4 CTAs/SM 0.1087-0.1104, pf4 at 3 CTAs/SM 0.1083-0.1088,
+    // unroll 2 0.1089, 64x8 0.111, 64x32 0.116, 64x16 with 4-row patches 0.1094
+    SDAG_STAR_PAIR(v, Jacobi7Star, "jacobi7", 64, 16, 2, 6, 0);
+    SDAG_STAR_PAIR(v, Jacobi7Star, "jacobi7", 64, 16, 2, 3, 6);
     SDAG_CROSS_PAIR(v, "jacobi7", 64, 8, 2, 3, 1);
     SDAG_CROSS_PAIR(v, "jacobi7", 64, 16, 4, 6, 2);
     SDAG_CROSS_PAIR(v, "jacobi7", 64, 8, 2, 6, 3);
     SDAG_CROSS_PAIR(v, "jacobi7", 64, 32, 4, 4, 4);
     SDAG_CROSS_PAIR(v, "jacobi7", 64, 64, 8, 3, 5);
-    SDAG_STAR_PAIR(v, Jacobi7Star, "jacobi7", 64, 16, 2, 6, 6);
     SDAG_PAIR(v, Jacobi7, "jacobi7", 64, 16, 1, 4, 2, 10);
     // temporal fusion for apply_iterated (NEXT-1; the paper's 7pt-smoother,
     // Table II): two sweeps per launch, overlapped tiles.  The cross stencil's

@@ -57,7 +57,7 @@ KernelDesc make_star_desc(const char *dag, int prio) {
     if (UNR > 1) std::snprintf(unr, sizeof unr, "_z%d", UNR);
     std::snprintf(buf, sizeof buf, "star%s_%s_%dx%d_u2x%d_pf%d%s%s",
                   QMODE == 1 ? "q" : (QMODE == 2 ? "DIFFmem" : (QMODE == 3 ? "DIFFnost" : (QMODE == 4 ? "L" : (QMODE == 5 ? "S" : (QMODE == 6 ? "R" : ""))))), TMA ? "tma" : "lsu", TX,
-                  TY, UY, PF, MINB > 1 ? (MINB == 2 ? "_mb2" : "_mb3") : "", unr);
+                  TY, UY, PF, MINB > 1 ? (MINB == 2 ? "_mb2" : (MINB == 3 ? "_mb3" : "_mb4")) : "", unr);
     d.variant = buf;
     d.fn = reinterpret_cast<const void *>(&dev::sdag_star<B, TX, TY, UY, PF, TMA, QMODE, MINB, UNR>);
     if constexpr (QMODE == 0)  // the dist p2p path's fused-store twin

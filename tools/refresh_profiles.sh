@@ -14,7 +14,7 @@ done
 # name -> ncu_counters key (variant@dims) of the kernel the plan picks
 declare -A KEY=(
   [lap25]="star_tma_32x32_u2x4_pf3_z2@512x512x512"
-  [jacobi7]="star_tma_64x16_u2x2_pf3@128x64x64x64"
+  [jacobi7]="star_tma_64x16_u2x2_pf6@128x64x64x64"
   [hypterm]="hyp_tma_64x8_u2x1_pf2@320x320x320"
   [rhs4center]="r4_tma_32x16_u2x1_pf1@320x320x320"
   [smooth27]="box_tma_128x16_u2x4_pf2@512x512x512"
