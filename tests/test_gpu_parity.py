@@ -58,6 +58,31 @@ def test_every_variant(name):
         check(name, dims, g, case)
 
 
+@pytest.mark.parametrize("name", NAMES)
+@pytest.mark.parametrize("dims", [(13, 22, 40), (11, 13, 35)], ids=["tma", "lsu"])
+def test_batched_every_dag(name, dims):
+    """sdag_apply_batched: B independent problems laid out [batch][nz][ny][nx]
+    (1D arrays [batch][len], include/sdag.h) in one launch; every problem
+    matches its own oracle and keeps its own ring (rhs4center's strx/stry/strz
+    are per problem, so a wrong 1D batch stride fails here)."""
+    B = 3
+    cases = [make_case(name, dims, cfg=f"batch{b}") for b in range(B)]
+    plan = sdag.Plan(sdag.spec_text(name), dims, batch=B)
+    dev = [torch.from_numpy(np.ascontiguousarray(np.stack([c["inputs"][q] for c in cases]))).cuda()
+           for q in range(len(cases[0]["inputs"]))]
+    if cases[0]["inout"]:
+        outs = [torch.from_numpy(np.stack([c["inout"][m] for c in cases])).cuda() for m in range(len(cases[0]["inout"]))]
+    else:
+        outs = [torch.full((B, *dims), np.nan, dtype=torch.float64, device="cuda") for _ in range(cases[0]["outs"])]
+    a1d = [torch.from_numpy(np.concatenate([c["a1d"][q] for c in cases])).cuda() for q in range(len(cases[0]["a1d"]))]
+    for c in cases[1:]:
+        assert c["s"] == cases[0]["s"], "scalars are shared by the batch"
+    plan.apply_batched(B, outs + dev, a1d, cases[0]["s"])
+    torch.cuda.synchronize()
+    for b, c in enumerate(cases):
+        check(name, dims, [t[b].cpu().numpy() for t in outs], c)
+
+
 def test_lsu_variants_on_odd_nx():
     dims = (11, 13, 35)
     for name in NAMES:
