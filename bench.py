@@ -197,19 +197,26 @@ def build_arrays(sdag, plan, name, dims, batch=1):
     return arrays3d, arrays1d, scal
 
 
-def timed(step, steps, warmup, stream, clock_index):
-    """W untimed steps, then K steps between CUDA events on `stream` (synchronised
-    on both sides), nvidia-smi clocks sampled during the timed region.
+def timed(step, steps, warmup, stream, clock_index, barrier=None):
+    """K steps between CUDA events on `stream`, max-over-ranks done by the caller.
+    The nvidia-smi clock sampler starts first (it needs ~0.3 s to come up); the W
+    warm-up steps run after it, right before the timed region, so the GPU enters
+    the region busy and at its working clocks rather than after 0.3 s idle (an
+    idle GPU adds ~0.1 ms of ramp to the first timed launch: a 10-step region of
+    the batched Jacobi read 0.117 ms per step, 100 steps 0.1066). Then a
+    synchronize, the ranks' barrier (N > 1), a synchronize, and the K steps.
     -> (ms per step, launches per step, clocks)"""
     import torch
     import paper_conf_ipps_rawatvsrps19_b200 as sdag
-    for _ in range(warmup):
-        step()
-    torch.cuda.synchronize()
-    l0 = sdag.launch_count()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with Clocks(clock_index) as clk:
+        for _ in range(warmup):
+            step()
         torch.cuda.synchronize()
+        if barrier is not None:
+            barrier()
+            torch.cuda.synchronize()
+        l0 = sdag.launch_count()
         e0.record(stream)
         for _ in range(steps):
             step()
@@ -445,8 +452,7 @@ def measure_config5_slabs(tdist, rank, world, local, steps, warmup, comm, halo="
         x1 = x0.clone()
         cs = torch.cuda.Stream()
         step = lambda: dd.apply_iterated(x0, x1, T, scalars=scal, stream=stream, comm_stream=cs)  # noqa: E731
-    tdist.barrier()
-    msN, lps, clk = timed(step, steps, warmup, stream, local)
+    msN, lps, clk = timed(step, steps, warmup, stream, local, barrier=tdist.barrier)
     t = torch.tensor([ms1, msN], dtype=torch.float64, device=_red_dev(halo))
     tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
     ms1m, msNm = float(t[0]), float(t[1])
@@ -601,8 +607,7 @@ def main():
         del src
         kplan = dd.plan
         info = kplan.info
-        tdist.barrier()
-        ms, lps, clk = timed(step, args.steps, args.warmup, stream, local)
+        ms, lps, clk = timed(step, args.steps, args.warmup, stream, local, barrier=tdist.barrier)
         t = torch.tensor([ms], dtype=torch.float64, device=rdev)
         tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
         ms = float(t[0])
@@ -677,7 +682,7 @@ def main():
             for cid in [x for x in args.configs.split(",") if x]:
                 # heuristic plans by default (deterministic variants, whose ncu counters are
                 # committed); --tune-configs times the plan-time measured pick instead
-                per[cid] = measure_config(cid, min(args.steps, 10), 3, peak_hbm, peak_src, fp64,
+                per[cid] = measure_config(cid, min(args.steps, 10) if cid == "5" else args.steps, 3, peak_hbm, peak_src, fp64,
                                           tune=args.tune_configs)
             per["fp64_peak_tflops_measured"] = fp64 / 1e12
         else:
