@@ -278,6 +278,14 @@ sdag_status sdag_nccl_get_unique_id(uint8_t id[128]);
 sdag_status sdag_nccl_comm_create(const uint8_t id[128], int32_t nranks, int32_t rank, int32_t device,
                                   void **comm);
 void sdag_nccl_comm_destroy(void *comm);
+/* Diagnostic: one NCCL group { ncclSend(send -> peer), ncclRecv(recv <- peer) }
+ * of `count` doubles on `stream`, through the same grouped call the z-slab halo
+ * exchange makes (error handling included).  `peer` may be this rank (a 1-rank
+ * communicator sends to itself), which lets a single GPU exercise the exact
+ * NCCL entry points, datatype and counts the exchange uses.  Device buffers,
+ * caller-owned; enqueued asynchronously. */
+sdag_status sdag_nccl_sendrecv(void *comm, int32_t peer, const double *send, double *recv, int64_t count,
+                               void *stream);
 
 /* SURVEY 8(b)'s form: this rank's slab from a LOCAL plan of its owned planes
  * (dims = nz_own, ny, nx), every rank owning nz_own planes (weak scaling:

@@ -23,7 +23,7 @@ from ._capi import PlanInfo, PlanOpts, SDAG_DEVICE_CURRENT, SDAG_DEVICE_NONE
 
 __all__ = ["Plan", "Program", "Dist", "SdagError", "registry", "spec_text", "fusion_schedule", "slab_partition", "slab_halo", "slab_partition2", "slab_halo2", "fission", "fuse_program", "program_version", "program_forest",
            "program_forest_tune", "nccl_unique_id",
-           "nccl_comm_create", "nccl_comm_destroy", "launch_count", "fp64_peak", "version", "SPEC_DIR"]
+           "nccl_comm_create", "nccl_comm_destroy", "nccl_sendrecv", "launch_count", "fp64_peak", "version", "SPEC_DIR"]
 
 SPEC_DIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "specs")
 
@@ -409,6 +409,18 @@ def nccl_comm_create(uid: bytes, nranks: int, rank: int, device: int) -> int:
 
 def nccl_comm_destroy(comm: int):
     _capi.lib().sdag_nccl_comm_destroy(ctypes.c_void_p(comm))
+
+
+def nccl_sendrecv(comm: int, peer: int, send, recv, stream=None):
+    """One grouped ncclSend(send -> peer) + ncclRecv(recv <- peer) through the halo
+    exchange's code path (sdag_nccl_sendrecv); peer may be this rank."""
+    if not send.is_contiguous() or not recv.is_contiguous():
+        raise TypeError("send and recv must be contiguous")
+    if send.numel() != recv.numel():
+        raise ValueError("send and recv must have the same number of elements")
+    _check(_capi.lib().sdag_nccl_sendrecv(ctypes.c_void_p(comm), int(peer), ctypes.c_void_p(_ptr(send, "send")),
+                                          ctypes.c_void_p(_ptr(recv, "recv")), int(send.numel()),
+                                          _stream_handle(stream)))
 
 
 class Dist:

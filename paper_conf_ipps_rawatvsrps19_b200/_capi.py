@@ -80,6 +80,7 @@ def lib():
             "sdag_nccl_get_unique_id": (S, [ctypes.c_char_p]),
             "sdag_nccl_comm_create": (S, [ctypes.c_char_p, c_i32, c_i32, c_i32, ctypes.POINTER(c_void_p)]),
             "sdag_nccl_comm_destroy": (None, [c_void_p]),
+            "sdag_nccl_sendrecv": (S, [c_void_p, c_i32, c_void_p, c_void_p, ctypes.c_int64, c_void_p]),
             "sdag_dist_create": (S, [c_char_p, c_i64p, ctypes.POINTER(PlanOpts), c_i32, c_i32, c_void_p,
                                      ctypes.POINTER(P)]),
             "sdag_dist_layout": (S, [P, c_i64p, c_i64p]),
@@ -144,7 +145,7 @@ EXPORTED = [
     "sdag_program_destroy",
     "sdag_apply_host", "sdag_fusion_schedule", "sdag_slab_partition", "sdag_slab_halo",
     "sdag_slab_partition2", "sdag_slab_halo2", "sdag_nccl_get_unique_id", "sdag_nccl_comm_create",
-    "sdag_nccl_comm_destroy", "sdag_dist_create", "sdag_dist_create_local", "sdag_dist_layout", "sdag_dist_alloc_dims", "sdag_dist_local_plan", "sdag_dist_apply",
+    "sdag_nccl_comm_destroy", "sdag_nccl_sendrecv", "sdag_dist_create", "sdag_dist_create_local", "sdag_dist_layout", "sdag_dist_alloc_dims", "sdag_dist_local_plan", "sdag_dist_apply",
     "sdag_dist_apply_iterated", "sdag_dist_destroy", "sdag_dist_apply_host", "sdag_dist_apply_iterated_loopback",
     "sdag_spec_fission", "sdag_program_version", "sdag_program_forest", "sdag_program_forest_tune", "sdag_program_fuse", "sdag_plan_profile", "sdag_dist_p2p_alloc", "sdag_dist_p2p_handle", "sdag_dist_p2p_attach", "sdag_dist_p2p_attach_local",
     "sdag_dist_p2p_apply_iterated", "sdag_last_error",

@@ -314,6 +314,11 @@ sdag_status sdag_nccl_comm_create(const uint8_t id[128], int32_t nranks, int32_t
 
 void sdag_nccl_comm_destroy(void *comm) { sdag::nccl_comm_destroy(comm); }
 
+sdag_status sdag_nccl_sendrecv(void *comm, int32_t peer, const double *send, double *recv, int64_t count,
+                               void *stream) {
+    return guard([&] { sdag::nccl_sendrecv(comm, peer, send, recv, count, reinterpret_cast<cudaStream_t>(stream)); });
+}
+
 sdag_status sdag_dist_create(const char *spec, const int64_t global_dims[3], const sdag_plan_opts *opts,
                              int32_t rank, int32_t nranks, void *nccl_comm, sdag_dist *out) {
     return guard([&] {

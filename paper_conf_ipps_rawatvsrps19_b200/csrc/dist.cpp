@@ -261,19 +261,19 @@ std::vector<int> halo_arrays(const Dist *d) {
     return v;
 }
 
-void exchange_nccl(Dist *d, double *const *a3, cudaStream_t comm, int planes) {
-    if (planes == 0 || d->nranks == 1) return;
-    if (!d->comm) throw Error(SDAG_ERR_INVALID_ARG, "multi-rank dist without an NCCL communicator");
+// One NCCL group of point-to-point transfers (send[i] -> peer[i], recv[i] <- peer[i]).
+// Every Send/Recv between GroupStart and GroupEnd is made even after a failure,
+// and GroupEnd always runs: an open group would corrupt every later call on the
+// communicator.  The first error is reported after the group is closed.
+struct Xfer {
+    const double *send;
+    double *recv;
+    size_t count;
+    int peer;
+};
+void nccl_group(void *comm, const std::vector<Xfer> &xs, cudaStream_t st) {
     const NcclApi &N = nccl();
-    const Plan *p = d->local;
-    const size_t plane = size_t(p->dims[1] * p->dims[2]);
-    const size_t cnt = plane * size_t(planes);
-    const Halo h = halo_schedule(d->slab, planes);
-    auto c = static_cast<ncclComm_t>(d->comm);
-    NvtxRange nr("sdag_halo_exchange_nccl");
-    // every call between GroupStart and GroupEnd is made even after a failure,
-    // and GroupEnd always runs: an open group would corrupt every later call on
-    // the communicator.  The first error is reported after the group is closed.
+    auto c = static_cast<ncclComm_t>(comm);
     ncclResult_t first = 0;
     const char *first_what = nullptr;
     auto call = [&](ncclResult_t r, const char *what) {
@@ -283,28 +283,50 @@ void exchange_nccl(Dist *d, double *const *a3, cudaStream_t comm, int planes) {
         }
     };
     nck(N.GroupStart(), "ncclGroupStart");
-    for (int f : halo_arrays(d)) {
-        double *a = a3[f];
-        if (h.lo_send >= 0) {
-            call(N.Send(a + size_t(h.lo_send) * plane, cnt, ncclFloat64, d->rank - 1, c, comm), "ncclSend");
-            call(N.Recv(a + size_t(h.lo_recv) * plane, cnt, ncclFloat64, d->rank - 1, c, comm), "ncclRecv");
-        }
-        if (h.up_send >= 0) {
-            call(N.Send(a + size_t(h.up_send) * plane, cnt, ncclFloat64, d->rank + 1, c, comm), "ncclSend");
-            call(N.Recv(a + size_t(h.up_recv) * plane, cnt, ncclFloat64, d->rank + 1, c, comm), "ncclRecv");
-        }
+    for (const Xfer &x : xs) {
+        call(N.Send(x.send, x.count, ncclFloat64, x.peer, c, st), "ncclSend");
+        call(N.Recv(x.recv, x.count, ncclFloat64, x.peer, c, st), "ncclRecv");
     }
     const ncclResult_t ge = N.GroupEnd();
     if (first != 0) nck(first, first_what);
     nck(ge, "ncclGroupEnd");
     // SDAG_NCCL_CHECK=1 (debug): poll the communicator's asynchronous error
-    // after every exchange (failure detection)
+    // after every group (failure detection)
     static const bool async_check = std::getenv("SDAG_NCCL_CHECK") && std::getenv("SDAG_NCCL_CHECK")[0] == '1';
     if (async_check && N.CommGetAsyncError) {
         ncclResult_t ae = 0;
         nck(N.CommGetAsyncError(c, &ae), "ncclCommGetAsyncError");
         nck(ae, "NCCL asynchronous error");
     }
+}
+
+}  // namespace
+
+void nccl_sendrecv(void *comm, int peer, const double *send, double *recv, int64_t count, cudaStream_t st) {
+    if (!comm) throw Error(SDAG_ERR_INVALID_ARG, "null communicator");
+    if (count < 0 || (count > 0 && (!send || !recv))) throw Error(SDAG_ERR_INVALID_ARG, "bad buffers");
+    nccl_group(comm, {Xfer{send, recv, size_t(count), peer}}, st);
+}
+
+namespace {
+
+void exchange_nccl(Dist *d, double *const *a3, cudaStream_t comm, int planes) {
+    if (planes == 0 || d->nranks == 1) return;
+    if (!d->comm) throw Error(SDAG_ERR_INVALID_ARG, "multi-rank dist without an NCCL communicator");
+    const Plan *p = d->local;
+    const size_t plane = size_t(p->dims[1] * p->dims[2]);
+    const size_t cnt = plane * size_t(planes);
+    const Halo h = halo_schedule(d->slab, planes);
+    NvtxRange nr("sdag_halo_exchange_nccl");
+    // to the lower neighbour: my lowest `planes` owned planes, its planes into my
+    // ghosts below; likewise above (halo_schedule, tested bitwise via loopback)
+    std::vector<Xfer> xs;
+    for (int f : halo_arrays(d)) {
+        double *a = a3[f];
+        if (h.lo_send >= 0) xs.push_back({a + size_t(h.lo_send) * plane, a + size_t(h.lo_recv) * plane, cnt, d->rank - 1});
+        if (h.up_send >= 0) xs.push_back({a + size_t(h.up_send) * plane, a + size_t(h.up_recv) * plane, cnt, d->rank + 1});
+    }
+    nccl_group(d->comm, xs, comm);
 }
 
 // local planes of the global z-interior (multi-sweep kernels keep the rest fixed)

@@ -86,5 +86,7 @@ void dist_p2p_apply_iterated(Dist *d, int T, const double *s, int ns, cudaStream
 void nccl_unique_id(uint8_t id[128]);
 void *nccl_comm_create(const uint8_t id[128], int nranks, int rank, int device);
 void nccl_comm_destroy(void *comm);
+// one grouped ncclSend + ncclRecv with `peer` (the halo exchange's code path; peer may be this rank)
+void nccl_sendrecv(void *comm, int peer, const double *send, double *recv, int64_t count, cudaStream_t st);
 
 }  // namespace sdag
