@@ -16,6 +16,9 @@ void add_kernels_hypterm(std::vector<KernelDesc> &v) {
     // round 2, measured and removed (ms at 320^3 vs 0.779 for 64x8 pf2): 32x16 pf2
     // 0.850 (less y-halo fill, fewer warps/SM), 32x8 pf3 1.046
     SDAG_HYP_PAIR(v, "hypterm", 32, 8, 2, 4);
+    // 12 warps/SM (64x12 or 32x24 tiles, 384 threads, pf1 to fit the ring) caps
+    // the thread at 168 registers: 896 B of spill stores per thread, into the
+    // shared/L1 data pipe that already binds this kernel -- not registered
     // round 2, measured and removed: plane loop unrolled 2 / 4 / 8 (the 8-slot
     // output ring rotated by register renaming instead of ~90 moves per plane):
     // 0.781-0.787 / 1.27 (spills) / 1.40 (spills) ms vs 0.778 -- the moves are
