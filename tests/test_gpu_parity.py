@@ -83,6 +83,50 @@ def test_batched_every_dag(name, dims):
         check(name, dims, [t[b].cpu().numpy() for t in outs], c)
 
 
+@pytest.mark.parametrize("name", ["jacobi7", "smooth27", "lap25"])
+def test_iterated_zero_sweeps_leaves_both_buffers(name):
+    """T = 0 (the degenerate iteration): nothing is launched, the result is buf0
+    as given and buf1 is untouched (bitwise)."""
+    dims = (14, 20, 36)
+    case = make_case(name, dims)
+    plan = sdag.Plan(sdag.spec_text(name), dims)
+    b0 = torch.from_numpy(case["inputs"][0].copy()).cuda()
+    b1 = torch.full(dims, np.nan, dtype=torch.float64, device="cuda")
+    l0 = sdag.launch_count()
+    plan.apply_iterated(b0, b1, 0, case["s"])
+    torch.cuda.synchronize()
+    assert sdag.launch_count() == l0
+    assert np.array_equal(b0.cpu().numpy(), case["inputs"][0])
+    assert np.all(np.isnan(b1.cpu().numpy()))
+
+
+def test_batch_beyond_the_launch_grid_is_refused():
+    """The largest batch one launch can carry: grid.z = z-chunks x batch <= 65535.
+    65535 one-plane problems run; 65536 are refused with DOMAIN before anything
+    is enqueued (the outputs keep their sentinel)."""
+    dims = (3, 3, 4)  # one interior point per problem
+    for B, ok in ((65535, True), (65536, False)):
+        plan = sdag.Plan(sdag.spec_text("jacobi7"), dims, batch=B)
+        A = torch.rand((B, *dims), dtype=torch.float64, device="cuda")
+        out = torch.full((B, *dims), np.nan, dtype=torch.float64, device="cuda")
+        if ok:
+            plan.apply_batched(B, [out, A], scalars=[4.0, 0.5, 0.25])
+            torch.cuda.synchronize()
+            a = A[:, 1, 1, 1:3].cpu().numpy()
+            nb = (A[:, 0, 1, 1:3] + A[:, 2, 1, 1:3] + A[:, 1, 0, 1:3] + A[:, 1, 2, 1:3]).cpu().numpy()
+            nb = nb + np.stack([A[:, 1, 1, 0].cpu().numpy(), A[:, 1, 1, 1].cpu().numpy()], 1) \
+                + np.stack([A[:, 1, 1, 2].cpu().numpy(), A[:, 1, 1, 3].cpu().numpy()], 1)
+            ref = 0.5 * a - (0.25 * 4.0) * (nb - 6.0 * a)
+            got = out[:, 1, 1, 1:3].cpu().numpy()
+            assert np.max(np.abs(got - ref) / np.maximum(np.abs(ref), 1.0)) < 1e-12
+        else:
+            with pytest.raises(sdag.SdagError) as e:
+                plan.apply_batched(B, [out, A], scalars=[4.0, 0.5, 0.25])
+            assert e.value.code == "DOMAIN"
+            torch.cuda.synchronize()
+            assert torch.all(torch.isnan(out))
+
+
 def test_lsu_variants_on_odd_nx():
     dims = (11, 13, 35)
     for name in NAMES:
