@@ -157,3 +157,17 @@ def test_full_smooth27_iterated_slabs_every_point(tune):
         g = res[z0:z1].cpu().numpy()
         gate(g, o, a, what=f"planes [{z0},{z1}) {plan.info['variant']}")
         del win, o, a, g
+
+
+@pytest.mark.parametrize("name", ["lap25", "hypterm", "rhs4center", "smooth27"])
+def test_large_ragged_every_point(name):
+    """A large grid ragged in every axis (no extent a multiple of any tile or
+    z-chunk; nx even so the TMA path runs): every interior point vs the oracle,
+    every ring point untouched -- the tile and chunk tails at scale."""
+    from cases import make_case, run_gpu, check
+    dims = {"lap25": (389, 262, 514), "hypterm": (211, 197, 302), "rhs4center": (203, 181, 266),
+            "smooth27": (401, 277, 390)}[name]
+    case = make_case(name, dims, cfg="ragged")
+    g, plan = run_gpu(name, dims, case)
+    assert "tma" in plan.info["variant"]
+    check(name, dims, g, case)
