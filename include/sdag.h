@@ -197,6 +197,7 @@ sdag_status sdag_program_stage(sdag_program prog, int32_t s, sdag_plan *out);
 sdag_status sdag_program_apply(sdag_program prog, int32_t batch, double *const *arrays3d, int32_t n3d,
                                const double *const *arrays1d, int32_t n1d, const double *scalars, int32_t nscalars,
                                sdag_stream stream);
+/* releases the program and its stage plans (their borrowed handles become invalid); NULL is a no-op */
 void sdag_program_destroy(sdag_program prog);
 
 /*
